@@ -1,0 +1,425 @@
+#!/usr/bin/env python
+"""Benchmark of the Jacobi halo/stencil hot path (BASELINE.json metric: "Jacobi GLUPS and % HBM
+roofline at 1/2/4/8 B200; halo hidden fraction").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--mode device|host] [--impl ours|reference]
+    torchrun --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N ...
+
+Workload (BASELINE.json configs[3], weak scaling): 16384 x 16384 fp32 points per GPU, ring in y
+(rank r owns rows r*16384..), device-initiated halo exchange fused into the stencil, the global
+L2 norm every 100 iterations.  At N = 1 this is also configs[2]'s single-GPU point.
+A "step" = one pass of the whole hot path: 100 Jacobi iterations (stencil + halo exchange on
+every iteration, the norm allreduce on the first), launched as one cached CUDA graph.
+GLUPS = NY * (NX - 2) * 100 * K / t / 1e9 over all ranks; t = max over ranks of the CUDA-event
+time of the K timed steps (inputs > L2: 2 GiB working set per GPU vs 126 MB L2, no flush needed).
+
+Timing protocol: barrier + synchronize on both sides of the timed region, W >= 3 warm-up steps.
+Extra objects on the JSON line: roofline (dominant kernel = jacobi_iter_kernel, per-launch CUDA
+events), cpu_baseline (the oracle on this host, rank 0, N = 1), e2e (host-buffer end-to-end through
+the C-ABI), clocks (nvidia-smi during the timed region), halo (exchange overlap).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "Jacobi GLUPS and % HBM roofline at 1/2/4/8 B200; halo hidden fraction"
+UNIT = "GLUPS"
+NX = 16384
+NY_PER_GPU = 16384
+ITERS_PER_STEP = 100
+NORM_EVERY = 100
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--mode", default="device", choices=["device", "host"])
+    ap.add_argument("--nx", type=int, default=NX)
+    ap.add_argument("--ny-per-gpu", type=int, default=NY_PER_GPU)
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--iters-per-step", type=int, default=ITERS_PER_STEP)
+    ap.add_argument("--norm-every", type=int, default=NORM_EVERY)
+    ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
+    ap.add_argument("--cpu-sample-iters", type=int, default=3)
+    ap.add_argument("--block-x", type=int, default=0)
+    ap.add_argument("--blocks-per-sm", type=int, default=0)
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def init_pg(rank, world):
+    import torch.distributed as dist
+    if world > 1 and not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+    return dist if world > 1 else None
+
+
+def allreduce_max(dist, x: float) -> float:
+    if dist is None:
+        return x
+    import torch
+    t = torch.tensor([x], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def barrier(dist):
+    if dist is not None:
+        dist.barrier()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def ncu_traffic(nx, n):
+    """Per-launch DRAM bytes of jacobi_iter_kernel from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    e = d.get(f"{nx}x{n}")
+    return None if e is None else float(e["dram_bytes_per_launch"])
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sms, maxs, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sms.append(float(f[1]))
+                maxs.append(float(f[2]))
+                power.append(float(f[3]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": max(maxs) if maxs else None,
+                "reasons": sorted(reasons), "samples": len(sms), "power_w_max": max(power) if power else None}
+
+
+# ----------------------------------------------------------------------------- our implementation
+def run_ours(a):
+    import numpy as np
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+
+    rank, world, local = dist_env()
+    if world != a.gpus:
+        raise SystemExit(f"--gpus {a.gpus} but WORLD_SIZE={world}")
+    dist = init_pg(rank, world)
+    torch.cuda.set_device(local)
+    ny = a.ny_per_gpu * world if a.scaling == "weak" else a.ny_per_gpu
+    nx = a.nx
+    mode = U.UC_MODE_DEVICE if a.mode == "device" else U.UC_MODE_HOST
+    env = U.Env(rank, world, local, U.torch_allgather() if world > 1 else None)
+    comm = U.Comm(env, *U.ring_neighbours(rank, world))
+    stream = torch.cuda.Stream()
+    coord = U.Coord(comm, mode, stream.cuda_stream)
+    J = U.Jacobi(comm, nx, ny)
+    if a.block_x or a.blocks_per_sm:
+        J.set_launch(a.block_x, a.blocks_per_sm)
+    n = J.n
+    launch_info = J.launch_info()
+    use_graph = not a.no_graph
+    ips = a.iters_per_step
+    pts_rank = n * (nx - 2)
+    norms_buf = np.zeros(max(1, ips // max(1, a.norm_every) + 1), np.float64)
+
+    def step():
+        J.run(coord, ips, a.norm_every, use_graph, norms_out=norms_buf)
+
+    for _ in range(a.warmup):
+        step()
+    coord.sync()
+
+    # ---------------- timed region: K steps, events on the coordinator's stream
+    clocks = ClockSampler(local)
+    barrier(dist)
+    torch.cuda.synchronize()
+    clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(a.steps):
+        step()
+    e1.record(stream)
+    coord.sync()
+    torch.cuda.synchronize()
+    barrier(dist)
+    clk = clocks.stop()
+    t_ms = e0.elapsed_time(e1)
+    t_max = allreduce_max(dist, t_ms)
+    ms_per_step = t_max / a.steps
+    total_pts = pts_rank * world * ips * a.steps
+    glups = total_pts / (t_max / 1e3) / 1e9
+    launches = a.steps * ips + (a.steps * ((ips + a.norm_every - 1) // a.norm_every) if a.mode == "host" else 0)
+
+    # ---------------- dominant kernel: per-launch events around single iterations (no norm / norm)
+    def kernel_ms(compute_norm, reps):
+        es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+        buf = np.zeros(1, np.float64)
+        for s, e in es:
+            s.record(stream)
+            J.step(coord, compute_norm, buf if compute_norm else None)
+            e.record(stream)
+        coord.sync()
+        return statistics.mean(s.elapsed_time(e) for s, e in es)
+
+    barrier(dist)
+    k_plain = allreduce_max(dist, kernel_ms(False, 50))
+    k_norm = allreduce_max(dist, kernel_ms(True, 10))
+    # the timed steps have 1 norm iteration per norm_every
+    nn = max(1, a.norm_every) if a.norm_every > 0 else ips
+    k_avg = (k_plain * (nn - 1) + k_norm) / nn
+    peak, peak_src = measured_peaks()
+    alg_bytes = 8.0 * pts_rank
+    achieved = alg_bytes / (k_plain / 1e3) / 1e9
+    roof = {"bound": "hbm", "kernel": "jacobi_iter_kernel", "achieved": round(achieved, 1), "peak": peak,
+            "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": ncu_traffic(nx, n),
+            "alg_bytes_per_launch": alg_bytes, "kernel_ms": round(k_plain, 5), "kernel_norm_ms": round(k_norm, 5),
+            "kernel_share_of_step": round(k_avg * ips / ms_per_step, 4), "peak_source": peak_src}
+
+    # ---------------- halo exchange overlap (differential, §8 d): same slab, no neighbours
+    halo = None
+    if not a.no_extras:
+        halo = halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_plain)
+
+    # ---------------- e2e through the C-ABI with pinned host buffers
+    e2e = None
+    if not a.no_extras:
+        slab_elems = (n + 2) * nx
+        h_in = torch.empty(slab_elems, dtype=torch.float32, pin_memory=True)
+        h_out = torch.empty(slab_elems, dtype=torch.float32, pin_memory=True)
+        h_norm = torch.zeros(8, dtype=torch.float64, pin_memory=True)
+        h_in.numpy()[:] = J.copy_out(coord).ravel()
+        ke = max(3, min(a.steps, 5))
+        barrier(dist)
+        torch.cuda.synchronize()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(ke):
+            J.copy_in_async(coord, h_in.data_ptr())
+            J.run(coord, ips, a.norm_every, use_graph, norms_out=h_norm.numpy())
+            J.copy_out_async(coord, h_out.data_ptr())
+        f1.record(stream)
+        coord.sync()
+        barrier(dist)
+        te = allreduce_max(dist, f0.elapsed_time(f1))
+        e2e = {"value": round(pts_rank * world * ips * ke / (te / 1e3) / 1e9, 3), "unit": UNIT,
+               "h2d_bytes_per_step": slab_elems * 4, "d2h_bytes_per_step": slab_elems * 4 + 8 * max(1, ips // nn),
+               "steps": ke, "ms_per_step": round(te / ke, 3)}
+
+    comm.barrier()
+    J.destroy()
+    coord.destroy()
+    comm.destroy()
+    env.finalize()
+
+    # ---------------- oracle on the host cores (rank 0, N = 1)
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_extras:
+        cpu = cpu_baseline(nx, a.ny_per_gpu, a.cpu_sample_iters)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(glups, 3), "unit": UNIT, "n_gpus": world, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+            "scaling": a.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"jacobi2d_{nx}x{a.ny_per_gpu}_per_gpu_{a.mode}_ring" if a.scaling == "weak"
+                       else f"jacobi2d_{nx}x{ny}_strong_{a.mode}_ring",
+                       "baseline_config": "configs[3] (weak, 16384^2 per GPU)" if a.scaling == "weak"
+                       else "configs[2] (strong, 16384^2 total)",
+                       "nx": nx, "ny_global": ny, "rows_per_gpu": n, "iters_per_step": ips,
+                       "norm_every": a.norm_every, "mode": a.mode, "cuda_graph": use_graph,
+                       "parallelism": f"y-slab x{world}", "l2": "inputs > L2 (2 slabs x "
+                       f"{(n + 2) * nx * 4 / 2**20:.0f} MiB per GPU vs 126 MB L2), no flush",
+                       "launch": launch_info},
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches,
+            "halo": halo, "pct_hbm_roofline": round(100 * glups / (world * peak / 8.0), 2),
+        }
+        print(json.dumps(line))
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full):
+    """hidden = clamp(1 - (T_full - T_compute) / T_xchg, 0, 1) (SURVEY §8 d).  T_compute: the same
+    slab and kernel with no neighbours (chain-less comm: top = bottom = -1 is not a valid Jacobi
+    topology for P > 1, so we time a P = 1 dirichlet-chain solver of the same n rows in its own
+    communicator); T_xchg: the exchange alone = put_signal of one row to each neighbour."""
+    # T_compute: independent single-rank chain (no waits, no puts) on this GPU
+    env1 = U.Env(0, 1, local)
+    comm1 = U.Comm(env1, -1, -1)
+    st = torch.cuda.Stream()
+    co1 = U.Coord(comm1, mode, st.cuda_stream)
+    J1 = U.Jacobi(comm1, nx, n)
+    es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(30)]
+    for s, e in es:
+        s.record(st)
+        J1.step(co1, False, None)
+        e.record(st)
+    co1.sync()
+    t_comp = statistics.mean(s.elapsed_time(e) for s, e in es[5:])
+    J1.destroy()
+    co1.destroy()
+    comm1.destroy()
+    env1.finalize()
+    t_full = k_full
+    # T_xchg: two row puts + signal waits (device mode), the same message size
+    comm = U.Comm(env, *U.ring_neighbours(rank, world))
+    st2 = torch.cuda.Stream()
+    co = U.Coord(comm, U.UC_MODE_DEVICE, st2.cuda_stream)
+    row = U.SymMem(comm, 2 * nx * 4)
+    sig = U.SymMem(comm, 256)
+    with torch.cuda.stream(st2):
+        src = torch.zeros(nx, dtype=torch.float32, device="cuda")
+    reps = 50
+    barrier(dist)
+    x0, x1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    x0.record(st2)
+    for i in range(1, reps + 1):
+        co.put_signal(src.data_ptr(), row, 0, nx * 4, sig, 0, i, comm.top)
+        co.put_signal(src.data_ptr(), row, nx * 4, nx * 4, sig, 16, i, comm.bottom)
+        co.signal_wait(row, 0, nx * 4, sig, 0, i, comm.bottom)
+        co.signal_wait(row, nx * 4, nx * 4, sig, 16, i, comm.top)
+    x1.record(st2)
+    co.sync()
+    t_x = x0.elapsed_time(x1) / reps
+    comm.barrier()
+    row.free()
+    sig.free()
+    co.destroy()
+    comm.destroy()
+    t_full = allreduce_max(dist, t_full)
+    t_comp = allreduce_max(dist, t_comp)
+    t_x = allreduce_max(dist, t_x)
+    hidden = max(0.0, min(1.0, 1.0 - (t_full - t_comp) / t_x)) if t_x > 0 else None
+    return {"hidden_fraction": None if hidden is None else round(hidden, 4), "t_full_ms": round(t_full, 5),
+            "t_compute_ms": round(t_comp, 5), "t_xchg_ms": round(t_x, 5),
+            "note": "per-iteration; t_xchg = standalone put_signal of both boundary rows + waits"}
+
+
+def cpu_baseline(nx, ny, iters):
+    """The oracle as it stands (single-threaded C, -O2), on a bounded sample of the workload."""
+    import oracle
+    from inputs import gen
+    oracle.build()
+    g = gen.global_field(nx, ny, "ring")
+    t = time.perf_counter()
+    oracle.jacobi_run(g, iters, "ring", 1)
+    dt = time.perf_counter() - t
+    return {"value": round(ny * (nx - 2) * iters / dt / 1e9, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{iters} iterations (norm every iteration) of the full {nx}x{ny} ring grid, "
+                      f"{dt:.1f} s, host {os.cpu_count()} cores visible, 1 used"}
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(a):
+    """The oracle (plain single-threaded C over the global grid) on the host cores, as the
+    reference arm: each step is a bounded sample (a.cpu_sample_iters... one iteration) of the
+    same 16384 x 16384-per-GPU workload."""
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    from inputs import gen
+    oracle.build()
+    nx, ny = a.nx, a.ny_per_gpu
+    g = gen.global_field(nx, ny, "ring")
+    iters = 1
+    for _ in range(a.warmup):
+        g, _s = oracle.jacobi_run(g, iters, "ring", 1)
+    t = time.perf_counter()
+    for _ in range(a.steps):
+        g, _s = oracle.jacobi_run(g, iters, "ring", 1)
+    dt = time.perf_counter() - t
+    v = ny * (nx - 2) * iters * a.steps / dt / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(dt / a.steps * 1e3, 2),
+            "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
+            "config": {"workload": f"jacobi2d_{nx}x{ny}_per_gpu_{a.mode}_ring", "nx": nx, "ny_global": ny,
+                       "sample": "1 iteration per step (norm each iteration) of the rank-0 grid"},
+            "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"{a.steps} steps x 1 iteration of {nx}x{ny}"},
+            "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+
+
+def main():
+    a = parse()
+    if a.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    if a.impl == "reference":
+        run_reference(a)
+    else:
+        run_ours(a)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,14 @@
+"""paper_conf_cluster_sagbilieinu25_b200 -- B200-native Jacobi halo/stencil hot path of UNICONN.
+
+The product is ``libuniconn_b200.so`` (C-ABI in ``include/uniconn.h``; CUDA for sm_100a in
+``csrc/``).  This package is its thin Python binding; importing it without the built library
+raises ImportError -- there is no CPU or PyTorch fallback.
+"""
+from .uniconn import (UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
+                      UC_TOPO_CHAIN, UC_TOPO_NONE, UC_TOPO_RING, UC_U64, Comm, Coord, Env, Jacobi, SymMem,
+                      ThreadAllgather, UCError, builtin_kernel, chain_neighbours, ring_neighbours,
+                      torch_allgather)
+from ._lib import EXPORTED, LIB_PATH, lib  # noqa: F401
+
+__all__ = ["Env", "Comm", "SymMem", "Coord", "Jacobi", "ThreadAllgather", "torch_allgather", "UCError",
+           "builtin_kernel", "ring_neighbours", "chain_neighbours", "lib", "LIB_PATH", "EXPORTED"]

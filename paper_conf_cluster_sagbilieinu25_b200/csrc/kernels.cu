@@ -1,0 +1,490 @@
+// kernels.cu -- sm_100a kernels of libuniconn_b200.
+//
+// The hot kernel is jacobi_iter_kernel: one Jacobi iteration k -> k+1 of a rank's slab
+// (§VI-C: 5-point 2-D star stencil, fp32, y-split), fused in device mode with
+// the halo exchange of Listing 3 (the blocks that compute the first and last rows put
+// them to the top/bottom neighbour and signal) and with the norm reduction (north_star).
+//
+// Design:
+//   * HBM-bound, 8 algorithmic bytes per updated point (4 B read of A_k, 4 B write of A_k+1).
+//   * One wave of blocks (grid = strips x chunks sized from occupancy); block (s, q) owns a
+//     strip of 4*blockDim columns (one float4 per thread) and a contiguous range of rows that
+//     it marches down in y, keeping rows y-1, y, y+1 in registers and prefetching the next
+//     kR rows (128-bit loads), so every point of A_k is read from HBM about once.
+//   * Left/right neighbours come from the adjacent lanes by warp shuffle; lanes 0/31 load the
+//     one scalar across the warp edge (an L1/L2 hit).
+//   * Device mode: block (s, 0) first computes row 1 (after waiting for the top neighbour's
+//     flag), stores it locally and straight into the top neighbour's halo row n+1 over NVLink,
+//     then release-sets the neighbour's per-strip flag; block (s, chunks-1) does the same for
+//     row n towards the bottom.  Only then do they march their interior rows, so the NVLink
+//     traffic overlaps the whole interior sweep (reading G10 for the flag protocol).
+//   * Norm iterations: d = new - old in fp32, d^2 accumulated in double per thread, warp
+//     shuffle + block reduction to one double per block; the last block (ticket) sums the
+//     block partials in index order, then (device mode) runs the one-shot cross-rank exchange.
+//   * The iteration counter lives on the device (k_dev[0]); the last block bumps it, so every
+//     launch has identical arguments and a CUDA graph of many iterations replays exactly.
+#include <cmath>
+
+#include "device_api.cuh"
+#include "uc_internal.h"
+
+namespace uc {
+using namespace dev;
+
+constexpr unsigned kFull = 0xffffffffu;
+constexpr int kR = 4;          // rows per prefetch batch
+constexpr int kMaxBlock = 256; // threads per block (upper bound)
+
+// ------------------------------------------------------------------------------ stencil math
+// Reading G1: new = 0.25f*((l+r)+(t+b)); __fadd_rn/__fmul_rn are never contracted into FMA
+// and do not flush subnormals (no --use_fast_math).
+__device__ __forceinline__ float upd(float l, float r, float t, float b) {
+  return __fmul_rn(0.25f, __fadd_rn(__fadd_rn(l, r), __fadd_rn(t, b)));
+}
+
+// New values of the 4 columns [4*x4, 4*x4+3] of row c, given the rows above (up) and below
+// (dn).  e is this lane's cross-warp neighbour: lane 0 holds column 4*x4-1, lane 31 holds
+// column 4*x4+4.  Columns 0 and NX-1 are Dirichlet (reading G2) and keep their value.
+// Must be called by all 32 lanes (shuffles).
+__device__ __forceinline__ float4 row_update(float4 up, float4 c, float4 dn, float e, int lane, int x4, int nx4) {
+  float L = __shfl_up_sync(kFull, c.w, 1);
+  float R = __shfl_down_sync(kFull, c.x, 1);
+  if (lane == 0) L = e;
+  if (lane == 31) R = e;
+  float4 o;
+  o.x = (x4 == 0) ? c.x : upd(L, c.y, up.x, dn.x);
+  o.y = upd(c.x, c.z, up.y, dn.y);
+  o.z = upd(c.y, c.w, up.z, dn.z);
+  o.w = (x4 == nx4 - 1) ? c.w : upd(c.z, R, up.w, dn.w);
+  return o;
+}
+
+__device__ __forceinline__ void acc_sq(double& acc, float4 o, float4 c) {
+  // d in fp32 (bit-identical to the oracle's d); (double)d*(double)d is exact.
+  const float d0 = __fsub_rn(o.x, c.x), d1 = __fsub_rn(o.y, c.y);
+  const float d2 = __fsub_rn(o.z, c.z), d3 = __fsub_rn(o.w, c.w);
+  acc += (double)d0 * (double)d0;
+  acc += (double)d1 * (double)d1;
+  acc += (double)d2 * (double)d2;
+  acc += (double)d3 * (double)d3;
+}
+
+// Read-only (non-coherent path) loads for rows that only this rank's previous kernel wrote.
+__device__ __forceinline__ float4 ld4_ro(const float* row, int x4, bool valid) {
+  return valid ? __ldg(reinterpret_cast<const float4*>(row) + x4) : make_float4(0.f, 0.f, 0.f, 0.f);
+}
+__device__ __forceinline__ float ld_edge_ro(const float* row, int x4, int lane, int nx4, bool valid) {
+  if (!valid) return 0.f;
+  if (lane == 0 && x4 > 0) return __ldg(row + 4 * x4 - 1);
+  if (lane == 31 && x4 + 1 < nx4) return __ldg(row + 4 * x4 + 4);
+  return 0.f;
+}
+// Coherent loads for the boundary rows (a neighbour may have just written the halo row).
+__device__ __forceinline__ float4 ld4_co(const float* row, int x4, bool valid) {
+  return valid ? reinterpret_cast<const float4*>(row)[x4] : make_float4(0.f, 0.f, 0.f, 0.f);
+}
+__device__ __forceinline__ float ld_edge_co(const float* row, int x4, int lane, int nx4, bool valid) {
+  if (!valid) return 0.f;
+  if (lane == 0 && x4 > 0) return row[4 * x4 - 1];
+  if (lane == 31 && x4 + 1 < nx4) return row[4 * x4 + 4];
+  return 0.f;
+}
+
+// ------------------------------------------------------------------------------ y-march
+// Computes rows y0..y1 (inclusive, slab coordinates) of dst from src for this thread's float4
+// column x4; reads rows y0-1..y1+1.  y0, y1 are block-uniform.
+template <bool NORM>
+__device__ __forceinline__ void march(const float* __restrict__ src, float* __restrict__ dst, int nx, int nx4,
+                                      int x4, int lane, int y0, int y1, double& acc) {
+  const bool valid = x4 < nx4;
+  const size_t pitch = (size_t)nx;
+  float4 up = ld4_ro(src + (size_t)(y0 - 1) * pitch, x4, valid);
+  float4 cur = ld4_ro(src + (size_t)y0 * pitch, x4, valid);
+  float ec = ld_edge_ro(src + (size_t)y0 * pitch, x4, lane, nx4, valid);
+  float4 nb[kR];
+  float ne[kR];
+#pragma unroll
+  for (int i = 0; i < kR; ++i) {
+    const int yy = y0 + 1 + i;
+    nb[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    ne[i] = 0.f;
+    if (yy <= y1 + 1) nb[i] = ld4_ro(src + (size_t)yy * pitch, x4, valid);
+    if (yy <= y1) ne[i] = ld_edge_ro(src + (size_t)yy * pitch, x4, lane, nx4, valid);
+  }
+  for (int y = y0; y <= y1; y += kR) {
+    // prefetch the next batch (rows y+kR+1 .. y+2kR) before consuming this one
+    float4 nn[kR];
+    float nne[kR];
+#pragma unroll
+    for (int i = 0; i < kR; ++i) {
+      const int yy = y + kR + 1 + i;
+      nn[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+      nne[i] = 0.f;
+      if (yy <= y1 + 1) nn[i] = ld4_ro(src + (size_t)yy * pitch, x4, valid);
+      if (yy <= y1) nne[i] = ld_edge_ro(src + (size_t)yy * pitch, x4, lane, nx4, valid);
+    }
+#pragma unroll
+    for (int i = 0; i < kR; ++i) {
+      if (y + i <= y1) {
+        const float4 dn = nb[i];
+        const float4 o = row_update(up, cur, dn, ec, lane, x4, nx4);
+        if (valid) __stcs(reinterpret_cast<float4*>(dst + (size_t)(y + i) * pitch) + x4, o);
+        if (NORM) acc_sq(acc, o, cur);
+        up = cur;
+        cur = dn;
+        ec = ne[i];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < kR; ++i) {
+      nb[i] = nn[i];
+      ne[i] = nne[i];
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------ boundary rows
+// Device mode: the fused compute + put + signal of one boundary row for strip s (Listing 3,
+// P:55-68; §8 a3).  top_side: row y == 1 goes to the top neighbour's halo row n+1;
+// bot_side: row y == n goes to the bottom neighbour's halo row 0.  Both when n == 1.
+template <bool NORM>
+__device__ __forceinline__ void boundary_row(const JacobiParams& p, const float* src, float* dst, int y, int x4,
+                                             int lane, int s, uint64_t k, bool top_side, bool bot_side,
+                                             double& acc) {
+  const bool put_top = top_side && p.has_top;
+  const bool put_bot = bot_side && p.has_bot;
+  if (threadIdx.x == 0) {
+    // halo rows of A_k (slab k&1) must hold the neighbours' A_k rows: wait for flag >= k
+    if (put_top) wait_ge(p.my_flags + (size_t)s * kFlagStride, k, p.timeout_ns, p.err);
+    if (put_bot) wait_ge(p.my_flags + (size_t)(p.strips + s) * kFlagStride, k, p.timeout_ns, p.err);
+  }
+  __syncthreads();
+  const bool valid = x4 < p.nx4;
+  const size_t pitch = (size_t)p.nx;
+  const float4 up = ld4_co(src + (size_t)(y - 1) * pitch, x4, valid);
+  const float4 cur = ld4_co(src + (size_t)y * pitch, x4, valid);
+  const float4 dn = ld4_co(src + (size_t)(y + 1) * pitch, x4, valid);
+  const float e = ld_edge_co(src + (size_t)y * pitch, x4, lane, p.nx4, valid);
+  const float4 o = row_update(up, cur, dn, e, lane, x4, p.nx4);
+  const int np = (int)((k + 1) & 1);
+  if (valid) {
+    reinterpret_cast<float4*>(dst + (size_t)y * pitch)[x4] = o;
+    // one-sided puts straight into the neighbours' halo rows of A_{k+1} over NVLink
+    if (put_top) reinterpret_cast<float4*>(p.top_slab[np] + (size_t)(p.n + 1) * pitch)[x4] = o;
+    if (put_bot) reinterpret_cast<float4*>(p.bot_slab[np])[x4] = o;
+  }
+  if (NORM) acc_sq(acc, o, cur);
+  if (put_top || put_bot) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence_system();
+      if (put_top) st_release_sys(p.top_flags + (size_t)(p.strips + s) * kFlagStride, k + 1);  // top's from_bottom[s]
+      if (put_bot) st_release_sys(p.bot_flags + (size_t)s * kFlagStride, k + 1);               // bottom's from_top[s]
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------ reductions
+__device__ __forceinline__ double block_sum(double v, double* smem) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  __syncthreads();
+  if (lane == 0) smem[w] = v;
+  __syncthreads();
+  double t = 0.0;
+  if (w == 0) {
+    t = lane < nw ? smem[lane] : 0.0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
+  }
+  return t;  // valid in thread 0
+}
+
+// Last block: deterministic sum of the block partials, cross-rank norm (device mode), counter bumps.
+__device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* smem) {
+  double tot = 0.0;
+  if (do_norm) {
+    double v = 0.0;
+    for (int i = threadIdx.x; i < (int)gridDim.x; i += blockDim.x) v += p.partials[i];
+    tot = block_sum(v, smem);
+  }
+  if (threadIdx.x == 0) {
+    if (do_norm) {
+      if (p.device_mode) {
+        // one-shot P2P allreduce of the rank partial (§8 a5): write slot[rank] on every rank,
+        // release a flag, wait for all P flags, sum slots 0..P-1 in rank order (reading G12).
+        const uint64_t m = p.k_dev[1];
+        const int par = (int)(m & 1);
+        for (int q = 0; q < p.size; ++q) st_relaxed_sys_f64(p.norm_slot[q] + par * p.size + p.rank, tot);
+        __threadfence_system();
+        for (int q = 0; q < p.size; ++q)
+          st_release_sys(p.norm_flag[q] + (size_t)(par * p.size + p.rank) * kFlagStride, m + 1);
+        double g = 0.0;
+        for (int q = 0; q < p.size; ++q) {
+          wait_ge(p.norm_flag[p.rank] + (size_t)(par * p.size + q) * kFlagStride, m + 1, p.timeout_ns, p.err);
+          g += ld_relaxed_sys_f64(p.norm_slot[p.rank] + par * p.size + q);
+        }
+        p.norm_hist[m % (uint64_t)p.norm_cap] = sqrt(g);
+        p.k_dev[1] = m + 1;
+      } else {
+        *p.rank_sum = tot;  // host mode: ncclAllReduce + norm_finish_kernel complete it
+      }
+    }
+    p.k_dev[0] = p.k_dev[0] + 1;
+    *p.done = 0;
+    __threadfence();
+  }
+}
+
+// ------------------------------------------------------------------------------ the kernel
+template <bool NORM>
+__device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t k) {
+  const int par = (int)(k & 1);
+  const float* src = p.slab[par];
+  float* dst = p.slab[par ^ 1];
+  const int s = blockIdx.x % p.strips;
+  const int q = blockIdx.x / p.strips;
+  const int lane = threadIdx.x & 31;
+  const int x4 = s * blockDim.x + threadIdx.x;
+  const int lo = 1 + (int)(((long long)q * p.n) / p.chunks);
+  const int hi = (int)(((long long)(q + 1) * p.n) / p.chunks);
+  double acc = 0.0;
+  int a = lo, b = hi;
+  if (p.device_mode) {
+    if (q == 0) boundary_row<NORM>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
+    if (q == p.chunks - 1 && p.n >= 2) boundary_row<NORM>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+    if (a < 2) a = 2;
+    if (b > p.n - 1) b = p.n - 1;
+  }
+  if (a <= b) march<NORM>(src, dst, p.nx, p.nx4, x4, lane, a, b, acc);
+  return acc;
+}
+
+__global__ void __launch_bounds__(kMaxBlock) jacobi_iter_kernel(const JacobiParams p) {
+  __shared__ double smem[kMaxBlock / 32];
+  __shared__ int s_last;
+  const uint64_t k = p.k_dev[0];
+  const bool do_norm = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
+  if (do_norm) {
+    const double acc = iteration_body<true>(p, k);
+    const double t = block_sum(acc, smem);
+    if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
+  } else {
+    iteration_body<false>(p, k);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned t = atomicAdd(p.done, 1u);
+    s_last = (t == gridDim.x - 1);
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    finish_iteration(p, do_norm, smem);
+  }
+}
+
+// Host mode: after ncclAllReduce of rank_sum, record sqrt into the history and bump m.
+__global__ void norm_finish_kernel(const double* rank_sum, double* norm_hist, int norm_cap,
+                                   unsigned long long* k_dev) {
+  const unsigned long long m = k_dev[1];
+  norm_hist[m % (unsigned long long)norm_cap] = sqrt(*rank_sum);
+  k_dev[1] = m + 1;
+}
+
+// ------------------------------------------------------------------------------ init
+__device__ __forceinline__ float hash_value(uint64_t seed, long long gy, int x, int nx) {
+  const uint64_t h = splitmix64(seed ^ ((uint64_t)gy * (uint64_t)nx + (uint64_t)x));
+  return (float)(h >> 40) * 0x1p-24f;  // 24-bit value, exact
+}
+
+__global__ void init_field_kernel(float* s0, float* s1, int nx, int n, int ny, int row0, int ring, uint64_t seed,
+                                  int zero_init, const float* colL, const float* toprow) {
+  const size_t total = (size_t)(n + 2) * nx;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
+    const int j = (int)(i / nx), x = (int)(i % nx);
+    const long long gy = (long long)row0 + j - 1;
+    float v;
+    if (ring) {
+      const long long gyw = ((gy % ny) + ny) % ny;
+      if (x == 0) v = colL[j];
+      else if (x == nx - 1) v = 0.f;
+      else v = zero_init ? 0.f : hash_value(seed, gyw, x, nx);
+    } else {
+      if (gy < 0) v = toprow[x];
+      else if (gy >= ny) v = 0.f;
+      else if (x == 0 || x == nx - 1) v = 0.f;
+      else v = zero_init ? 0.f : hash_value(seed, gy, x, nx);
+    }
+    s0[i] = v;
+    s1[i] = v;
+  }
+}
+
+// ------------------------------------------------------------------------------ P2P primitives
+// Post (one-sided, device mode): SM stores into the peer's buffer over NVLink, then the last
+// block release-stores the peer's signal (put_signal).
+__global__ void put_signal_kernel(const uint4* __restrict__ src, uint4* dst, size_t n16, const uint8_t* srcb,
+                                  uint8_t* dstb, size_t tail_off, size_t tail, uint64_t* sig, uint64_t val,
+                                  unsigned int* counter) {
+  const size_t stride = (size_t)gridDim.x * blockDim.x;
+  size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+  for (; i + 3 * stride < n16; i += 4 * stride) {
+    const uint4 a = src[i], b = src[i + stride], c = src[i + 2 * stride], d = src[i + 3 * stride];
+    dst[i] = a;
+    dst[i + stride] = b;
+    dst[i + 2 * stride] = c;
+    dst[i + 3 * stride] = d;
+  }
+  for (; i < n16; i += stride) dst[i] = src[i];
+  if (blockIdx.x == 0)
+    for (size_t t = threadIdx.x; t < tail; t += blockDim.x) dstb[tail_off + t] = srcb[tail_off + t];
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence_system();
+    const unsigned t = atomicAdd(counter, 1u);
+    if (t == gridDim.x - 1) {
+      *counter = 0;
+      __threadfence_system();
+      if (sig) st_release_sys(sig, val);
+    }
+  }
+}
+
+// Acknowledge (one-sided, device mode): the stream waits until the local signal >= val.
+__global__ void signal_wait_kernel(const uint64_t* sig, uint64_t val, unsigned long long timeout_ns,
+                                   unsigned int* err) {
+  if (threadIdx.x == 0) wait_ge(sig, val, timeout_ns, err);
+}
+
+struct PeerPtrs {
+  void* p[UC_MAX_RANKS];
+};
+struct PeerFlags {
+  uint64_t* p[UC_MAX_RANKS];
+};
+
+template <typename T>
+__device__ void oneshot_body(const T* send, T* recv, size_t count, int rank, int size, const PeerPtrs& slots,
+                             const PeerFlags& flags, const uint64_t* my_flags, const char* my_slots,
+                             uint64_t epoch, size_t slot_bytes, unsigned long long timeout_ns, unsigned int* err) {
+  const int par = (int)(epoch & 1);
+  for (int q = 0; q < size; ++q) {
+    T* dst = reinterpret_cast<T*>(static_cast<char*>(slots.p[q]) + (size_t)(par * size + rank) * slot_bytes);
+    for (size_t i = threadIdx.x; i < count; i += blockDim.x) dst[i] = send[i];
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence_system();
+    for (int q = 0; q < size; ++q) st_release_sys(flags.p[q] + (size_t)(par * size + rank) * kFlagStride, epoch);
+    for (int q = 0; q < size; ++q)
+      wait_ge(my_flags + (size_t)(par * size + q) * kFlagStride, epoch, timeout_ns, err);
+  }
+  __syncthreads();
+  for (size_t i = threadIdx.x; i < count; i += blockDim.x) {
+    T acc = T(0);
+    for (int q = 0; q < size; ++q) {
+      const volatile T* src =
+          reinterpret_cast<const volatile T*>(my_slots + (size_t)(par * size + q) * slot_bytes);
+      acc = acc + src[i];
+    }
+    recv[i] = acc;
+  }
+}
+
+__global__ void allreduce_oneshot_kernel(const void* send, void* recv, size_t count, int dtype, int rank, int size,
+                                         PeerPtrs slots, PeerFlags flags, const uint64_t* my_flags,
+                                         const char* my_slots, uint64_t epoch, size_t slot_bytes,
+                                         unsigned long long timeout_ns, unsigned int* err) {
+  if (dtype == UC_F32)
+    oneshot_body<float>((const float*)send, (float*)recv, count, rank, size, slots, flags, my_flags, my_slots, epoch,
+                        slot_bytes, timeout_ns, err);
+  else if (dtype == UC_F64)
+    oneshot_body<double>((const double*)send, (double*)recv, count, rank, size, slots, flags, my_flags, my_slots,
+                         epoch, slot_bytes, timeout_ns, err);
+  else
+    oneshot_body<unsigned long long>((const unsigned long long*)send, (unsigned long long*)recv, count, rank, size,
+                                     slots, flags, my_flags, my_slots, epoch, slot_bytes, timeout_ns, err);
+}
+
+// ------------------------------------------------------------------------------ launchers
+int launch_jacobi_iteration(const JacobiParams& p, int block, cudaStream_t s) {
+  jacobi_iter_kernel<<<p.strips * p.chunks, block, 0, s>>>(p);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev, int,
+                       cudaStream_t s) {
+  norm_finish_kernel<<<1, 1, 0, s>>>(rank_sum, norm_hist, norm_cap, k_dev);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int launch_init_field(float* slab0, float* slab1, int nx, int n, int ny, int row0, int ring, int, int, uint64_t seed,
+                      int zero_init, const float* colL, const float* toprow, cudaStream_t s) {
+  const size_t total = (size_t)(n + 2) * nx;
+  const int blocks = (int)std::min<size_t>((total + 255) / 256, 148 * 16);
+  init_field_kernel<<<blocks, 256, 0, s>>>(slab0, slab1, nx, n, ny, row0, ring, seed, zero_init, colL, toprow);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int launch_put_signal(const void* src, void* dst, size_t bytes, uint64_t* sig, uint64_t val, unsigned int* counter,
+                      cudaStream_t s) {
+  const size_t n16 = bytes / 16;
+  const size_t tail_off = n16 * 16, tail = bytes - tail_off;
+  size_t blocks = bytes / 32768;
+  if (blocks < 1) blocks = 1;
+  if (blocks > 296) blocks = 296;
+  put_signal_kernel<<<(unsigned)blocks, 256, 0, s>>>((const uint4*)src, (uint4*)dst, n16, (const uint8_t*)src,
+                                                     (uint8_t*)dst, tail_off, tail, sig, val, counter);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int launch_signal_wait(const uint64_t* sig, uint64_t val, unsigned long long timeout_ns, unsigned int* err,
+                       cudaStream_t s) {
+  signal_wait_kernel<<<1, 32, 0, s>>>(sig, val, timeout_ns, err);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dtype, int rank, int size,
+                             void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
+                             const void* my_slots, uint64_t epoch, size_t slot_bytes, unsigned long long timeout_ns,
+                             unsigned int* err, cudaStream_t s) {
+  PeerPtrs sp{};
+  PeerFlags fp{};
+  for (int q = 0; q < size; ++q) {
+    sp.p[q] = peer_slots[q];
+    fp.p[q] = peer_flags[q];
+  }
+  allreduce_oneshot_kernel<<<1, 256, 0, s>>>(send, recv, count, dtype, rank, size, sp, fp, my_flags,
+                                             (const char*)my_slots, epoch, slot_bytes, timeout_ns, err);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int jacobi_occupancy(int block, int* blocks_per_sm) {
+  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel, block, 0));
+  return UC_OK;
+}
+
+}  // namespace uc
+
+// Library kernel exposed for uc_launch tests (BindKernel/LaunchKernel of a user kernel).
+extern "C" __global__ void uc_fill_f32(float* dst, unsigned long long n, float value) {
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    dst[i] = value;
+}
+
+namespace uc {
+const void* builtin_kernel(const char* name) {
+  if (name && std::string(name) == "uc_fill_f32") return (const void*)uc_fill_f32;
+  return nullptr;
+}
+}  // namespace uc

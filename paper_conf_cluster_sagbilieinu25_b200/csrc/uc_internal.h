@@ -1,0 +1,170 @@
+// Internal definitions of libuniconn_b200 (not part of the C-ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cstdint>
+#include <algorithm>
+#include <cstdio>
+#include <string>
+#include <vector>
+
+#include "uniconn.h"
+
+namespace uc {
+
+// ----------------------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+int fail(int status, const char* fmt, ...);
+
+#define UC_CUDA(call)                                                                        \
+  do {                                                                                       \
+    cudaError_t uc_e_ = (call);                                                              \
+    if (uc_e_ != cudaSuccess)                                                                \
+      return ::uc::fail(UC_ERR_CUDA, "%s failed at %s:%d: %s", #call, __FILE__, __LINE__,     \
+                        cudaGetErrorString(uc_e_));                                          \
+  } while (0)
+
+#define UC_NCCL(call)                                                                        \
+  do {                                                                                       \
+    ncclResult_t uc_n_ = (call);                                                             \
+    if (uc_n_ != ncclSuccess)                                                                \
+      return ::uc::fail(UC_ERR_NCCL, "%s failed at %s:%d: %s", #call, __FILE__, __LINE__,     \
+                        ncclGetErrorString(uc_n_));                                          \
+  } while (0)
+
+#define UC_TRY(call)                                                                         \
+  do {                                                                                       \
+    int uc_s_ = (call);                                                                      \
+    if (uc_s_ != UC_OK) return uc_s_;                                                        \
+  } while (0)
+
+// ----------------------------------------------------------------------------- device-side shared structs
+// Everything a device-mode Jacobi iteration needs, passed by value to the kernel.
+struct JacobiParams {
+  float* slab[2];          // local ping-pong slabs, (n+2) x nx each
+  float* top_slab[2];      // top neighbour's slabs (nullptr when none)
+  float* bot_slab[2];      // bottom neighbour's slabs
+  uint64_t* my_flags;      // local: [0, S) from_top[s], [S, 2S) from_bottom[s] (stride kFlagStride)
+  uint64_t* top_flags;     // top neighbour's flag array (we set its from_bottom[s])
+  uint64_t* bot_flags;     // bottom neighbour's flag array (we set its from_top[s])
+  double* norm_slot[UC_MAX_RANKS];     // rank q's norm slots: [2][P] doubles
+  uint64_t* norm_flag[UC_MAX_RANKS];   // rank q's norm flags: [2][P] u64 (stride kFlagStride)
+  unsigned long long* k_dev;           // local iteration counter
+  unsigned int* done;                  // local block ticket
+  double* partials;                    // local [grid] per-block partial sums
+  double* rank_sum;                    // local: this rank's sum of squares (host-mode allreduce in place)
+  double* norm_hist;                   // local: norms by round m (ring of norm_cap)
+  unsigned int* err;                   // local error word (bit 0 = timeout)
+  unsigned long long timeout_ns;
+  int nx, n;               // columns, owned rows
+  int nx4;                 // nx / 4
+  int strips, chunks;      // grid = strips * chunks blocks
+  int has_top, has_bot;
+  int device_mode;         // 1: fused waits + puts + in-kernel cross-rank norm
+  int norm_every;          // <= 0: never
+  int norm_cap;
+  int rank, size;
+};
+
+constexpr int kFlagStride = 16;  // u64 per flag = 128 bytes, one flag per L2 line
+
+// Launch wrappers implemented in kernels.cu
+int launch_jacobi_iteration(const JacobiParams& p, int block, cudaStream_t s);
+int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
+                       int norm_every, cudaStream_t s);
+int launch_init_field(float* slab0, float* slab1, int nx, int n, int ny, int row0, int ring,
+                      int has_top, int has_bot, uint64_t seed, int zero_init, const float* colL,
+                      const float* toprow, cudaStream_t s);
+int launch_put_signal(const void* src, void* dst, size_t bytes, uint64_t* sig, uint64_t val,
+                      unsigned int* counter, cudaStream_t s);
+int launch_signal_wait(const uint64_t* sig, uint64_t val, unsigned long long timeout_ns, unsigned int* err,
+                       cudaStream_t s);
+int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dtype, int rank, int size,
+                             void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
+                             const void* my_slots, uint64_t epoch, size_t slot_bytes,
+                             unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
+int jacobi_occupancy(int block, int* blocks_per_sm);
+const void* builtin_kernel(const char* name);
+
+}  // namespace uc
+
+// ----------------------------------------------------------------------------- opaque handles
+struct uc_env {
+  int rank = 0, size = 1, device = 0;
+  uc_allgather_fn ag = nullptr;
+  void* ag_ctx = nullptr;
+  int live_comms = 0;
+  int allgather(const void* send, void* recv, size_t bytes);
+};
+
+struct PeerRecord {
+  uint64_t host_hash;
+  int32_t pid;
+  int32_t device;
+  int32_t top, bottom;
+  int32_t rank;
+  int32_t pad;
+};
+
+struct uc_comm {
+  uc_env* env = nullptr;
+  int rank = 0, size = 1, top = -1, bottom = -1;
+  int topology = UC_TOPO_NONE;
+  std::vector<PeerRecord> peers;
+  int* dev_view = nullptr;  // {rank, size, top, bottom}
+  int live_objects = 0;
+  bool same_process(int r) const;
+};
+
+struct uc_mem {
+  uc_comm* comm = nullptr;
+  size_t bytes = 0;
+  void* local = nullptr;
+  std::vector<void*> ptrs;      // per rank
+  std::vector<bool> ipc_opened; // per rank: close with cudaIpcCloseMemHandle
+};
+
+struct uc_coord {
+  uc_comm* comm = nullptr;
+  uc_mode mode = UC_MODE_HOST;
+  cudaStream_t stream = nullptr;
+  ncclComm_t nccl = nullptr;
+  int in_group = 0;
+  unsigned long long timeout_ns = 10ull * 1000 * 1000 * 1000;
+  unsigned int* err = nullptr;         // device error word
+  unsigned int* put_counter = nullptr; // device counter for multi-block put_signal
+  uc_mem* ar_scratch = nullptr;        // device-mode allreduce slots [2][P][slot_bytes] + flags
+  size_t ar_slot_bytes = 32768;
+  uint64_t ar_epoch = 0;
+  int live_jacobi_users = 0;
+};
+
+struct JacobiGraph {
+  int iters = 0, norm_every = 0, parity = 0, mode = -1;
+  cudaStream_t stream = nullptr;
+  cudaGraphExec_t exec = nullptr;
+};
+
+struct uc_jacobi {
+  uc_comm* comm = nullptr;
+  int nx = 0, n = 0, ny = 0, row0 = 0;
+  int ring = 0;
+  int64_t k = 0;                 // host mirror of the device iteration counter k_dev[0]
+  int64_t m = 0;                 // host mirror of the device norm-round counter k_dev[1]
+  uc_mem* slabs = nullptr;       // symmetric: 2 * (n+2) * nx floats
+  uc_mem* ctrl = nullptr;        // symmetric: flags + norm slots
+  size_t slab_elems = 0;
+  int strips = 0;
+  // local device state
+  unsigned long long* k_dev = nullptr;
+  unsigned int* done = nullptr;
+  double* partials = nullptr;
+  double* rank_sum = nullptr;
+  double* norm_hist = nullptr;
+  int norm_cap = 4096;
+  int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
+  int partials_cap = 0;
+  std::vector<JacobiGraph> graphs;
+};

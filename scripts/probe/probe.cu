@@ -39,9 +39,11 @@ __global__ void spin_until(const unsigned long long* flag, unsigned long long v,
 }
 __global__ void set_flag(unsigned long long* flag, unsigned long long v) { st_rel(flag, v); }
 
-int main() {
-  // ---------------- IPC + cross-process spin (fork before CUDA init)
+int main(int argc, char** argv) {
+  setvbuf(stdout, NULL, _IONBF, 0);
+  bool do_ipc = argc > 1 && !strcmp(argv[1], "ipc");
   int p2c[2], c2p[2];
+  if (do_ipc) {
   if (pipe(p2c) || pipe(c2p)) return 1;
   pid_t pid = fork();
   if (pid == 0) {
@@ -82,6 +84,11 @@ int main() {
     else printf("cross-process spin: saw flag after %.3f ms (child sleeps 200 ms first)\n", *out / 1e6);
   }
   int st; waitpid(pid, &st, 0);
+  return 0;
+  }
+  CK(cudaSetDevice(0));
+  { cudaDeviceProp prop; CK(cudaGetDeviceProperties(&prop, 0));
+  printf("device %s SMs=%d L2=%d MB\n", prop.name, prop.multiProcessorCount, prop.l2CacheSize >> 20); }
 
   // ---------------- copy bandwidth
   size_t n = (size_t)1 << 28;  // 1 GiB of floats

@@ -1,0 +1,82 @@
+"""Runs the CUDA path through the C-ABI for P virtual ranks on one GPU and assembles the
+global field, so tests can compare it with the oracle element by element."""
+from __future__ import annotations
+
+import numpy as np
+
+from inputs import gen
+from vranks import run_ranks
+
+MODES = {"device": 1, "host": 0}
+
+
+def neighbours(U, topology):
+    return U.ring_neighbours if topology == "ring" else U.chain_neighbours
+
+
+def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0, seed=gen.DEFAULT_SEED,
+              zero_init=False, init=None, use_graph=True, stepwise=False, block_x=0, blocks_per_sm=0,
+              chunks_of_run=None):
+    """Returns dict(init=[slab0 per rank], final=[slab per rank], norms=np.array (rank 0),
+    norms_all=[per rank], launch=launch_info of rank 0)."""
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+
+    def body(rank, P, ag):
+        env = U.Env(rank, P, 0, ag)
+        top, bot = neighbours(U, topology)(rank, P)
+        comm = U.Comm(env, top, bot)
+        stream = torch.cuda.Stream()
+        coord = U.Coord(comm, MODES[mode], stream.cuda_stream)
+        coord.set_timeout(30.0)
+        J = U.Jacobi(comm, nx, ny, seed, zero_init)
+        try:
+            if block_x or blocks_per_sm:
+                J.set_launch(block_x, blocks_per_sm)
+            slab0 = J.copy_out()
+            if init is not None:
+                J.copy_in(gen.rank_slab(init, rank, P))
+            if stepwise:
+                norms = []
+                for i in range(iters):
+                    want = norm_every > 0 and J.iteration % norm_every == 0
+                    buf = np.zeros(1, np.float64)
+                    J.step(coord, want, buf if want else None)
+                    coord.sync()
+                    if want:
+                        norms.append(buf[0])
+                norms = np.array(norms)
+            else:
+                parts = chunks_of_run or [iters]
+                outs = [J.run(coord, it, norm_every, use_graph) for it in parts]
+                coord.sync()
+                norms = np.concatenate(outs) if outs else np.zeros(0)
+            coord.sync()
+            final = J.copy_out(coord)
+            info = J.launch_info()
+            return slab0, final, norms, info
+        finally:
+            comm.barrier()
+            J.destroy()
+            coord.destroy()
+            comm.destroy()
+            env.finalize()
+
+    res = run_ranks(P, body)
+    return {"init": [r[0] for r in res], "final": [r[1] for r in res], "norms": res[0][2],
+            "norms_all": [r[2] for r in res], "launch": res[0][3]}
+
+
+def bits(a):
+    return np.ascontiguousarray(a, dtype=np.float32).view(np.uint32)
+
+
+def assert_slabs_equal_global(slabs, g, P, topology, what="final"):
+    for r, s in enumerate(slabs):
+        want = gen.rank_slab(g, r, P, topology)
+        if not np.array_equal(bits(s), bits(want)):
+            diff = np.argwhere(bits(s) != bits(want))
+            j, i = diff[0]
+            raise AssertionError(f"{what}: rank {r} differs at {len(diff)} points, first (row {j}, col {i}): "
+                                 f"gpu={s[j, i]!r} oracle={want[j, i]!r}")

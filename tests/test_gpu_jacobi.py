@@ -1,0 +1,149 @@
+"""GPU parity of the Jacobi hot path (C-ABI -> sm_100a kernels) against the CPU oracle.
+
+Bar (BASELINE.json north_star): the fp32 grid bit-exact after N iterations; the norm within
+1e-5 relative (reduction order differs; reading G12).  Multi-rank cases run as virtual ranks
+(threads, one GPU): the device-mode put/signal protocol runs for real, peers in one process.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from gpu_harness import assert_slabs_equal_global, bits, solve_gpu
+from inputs import gen
+
+pytestmark = pytest.mark.gpu
+
+NORM_RTOL = 1e-5
+
+
+def _oracle(nx, ny, topology, iters, norm_every, seed=gen.DEFAULT_SEED, zero_init=False, init=None):
+    g = init if init is not None else gen.global_field(nx, ny, topology, seed, zero_init)
+    out, sums = oracle.jacobi_run(g, iters, topology, norm_every)
+    return g, out, np.sqrt(sums)
+
+
+def _check(nx, ny, P, topology, mode, iters, norm_every=0, **kw):
+    init = kw.pop("init", None)
+    g0, want, want_norms = _oracle(nx, ny, topology, iters, norm_every, kw.get("seed", gen.DEFAULT_SEED),
+                                   kw.get("zero_init", False), init)
+    res = solve_gpu(nx, ny, P, topology, mode, iters, norm_every, init=init, **kw)
+    if init is None:
+        assert_slabs_equal_global(res["init"], g0, P, topology, "iteration 0 (generator parity)")
+    assert_slabs_equal_global(res["final"], want, P, topology)
+    assert len(res["norms"]) == len(want_norms)
+    for r_norms in res["norms_all"]:  # every rank holds the same norms, bit for bit
+        assert np.array_equal(r_norms, res["norms"])
+    for a, b in zip(res["norms"], want_norms):
+        assert a == b or abs(a - b) <= NORM_RTOL * abs(b), (a, b)
+    return res
+
+
+# --------------------------------------------------------------------------- C1 and shapes
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+@pytest.mark.parametrize("mode", ["device", "host"])
+def test_c1_256_100_iterations(topology, mode):
+    """BASELINE.json configs[0]: 256x256 fp32, 100 iterations, 1 GPU vs the oracle, bit-exact."""
+    _check(256, 256, 1, topology, mode, 100, norm_every=10)
+
+
+@pytest.mark.parametrize("nx,ny,iters", [(4, 2, 3), (8, 7, 20), (12, 5, 9), (1028, 64, 37), (2052, 33, 12),
+                                         (4096, 40, 8)])
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+def test_ragged_shapes_single_rank(nx, ny, iters, topology):
+    """Several strips with a ragged last strip (NX/4 not a multiple of the block), tiny grids,
+    odd row counts."""
+    _check(nx, ny, 1, topology, "device", iters, norm_every=4)
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+def test_partition_invariance_device_mode(P, topology):
+    """Virtual ranks: P = 2..8 give the oracle's global grid bit for bit (invariant 6)."""
+    _check(520, 24 * P, P, topology, "device", 25, norm_every=5)
+
+
+@pytest.mark.parametrize("P,ny", [(2, 2), (4, 4), (3, 3), (2, 4)])
+def test_one_or_two_rows_per_rank(P, ny):
+    """n = 1 (one row does both boundary sides) and n = 2; P = 2 has top == bottom."""
+    for topology in ("ring", "dirichlet"):
+        _check(64, ny, P, topology, "device", 11, norm_every=2)
+
+
+def test_host_mode_single_rank_nccl_self_exchange():
+    _check(1028, 50, 1, "ring", "host", 13, norm_every=3)
+
+
+def test_graph_and_stepwise_agree():
+    a = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=True)
+    b = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=False)
+    c = solve_gpu(516, 64, 2, "ring", "device", 30, 1, stepwise=True)
+    d = solve_gpu(516, 64, 2, "ring", "device", 30, 7, chunks_of_run=[3, 11, 16])
+    for x in (b, c, d):
+        for s1, s2 in zip(a["final"], x["final"]):
+            assert np.array_equal(bits(s1), bits(s2))
+    assert np.array_equal(a["norms"], b["norms"]) and np.array_equal(a["norms"], d["norms"])
+    assert np.array_equal(a["norms"], c["norms"][[0, 7, 14, 21, 28]])
+
+
+@pytest.mark.parametrize("block_x,bps", [(32, 1), (64, 2), (128, 0), (256, 1)])
+def test_launch_geometries(block_x, bps):
+    """Different block widths / chunk counts change blocking, not results."""
+    res = _check(1024, 96, 1, "ring", "device", 9, norm_every=3, block_x=block_x, blocks_per_sm=bps)
+    assert res["launch"]["block"] == block_x
+
+
+# --------------------------------------------------------------------------- pinned examples
+def _hand4x4(golden_dir):
+    rows = [l.split()[1:] for l in open(f"{golden_dir}/hand4x4.txt") if l.startswith("init")]
+    return np.array(rows, dtype=np.float32)
+
+
+@pytest.mark.parametrize("P,mode", [(1, "device"), (2, "device"), (1, "host")])
+def test_hand_worked_4x4(golden_dir, P, mode):
+    g = _hand4x4(golden_dir)
+    res = solve_gpu(4, 2, P, "dirichlet", mode, 3, 1, init=g)
+    got = np.vstack([s[1:-1] for s in res["final"]])
+    assert np.array_equal(got[:, 1:3], np.array([[4.53125, 6.25], [8.75, 13.28125]], np.float32))
+    want = [math.sqrt(132.8125), math.sqrt(22.8515625), math.sqrt(5.712890625)]
+    assert list(res["norms"]) == want  # dyadic sums: exact in any order
+
+
+def test_subnormal_front_no_ftz():
+    """4^-k front reaches subnormals (2^-128 .. 2^-148) bit-exactly: no FTZ on the GPU."""
+    nx, ny = 96, 4
+    a = np.zeros((ny + 2, nx), np.float32)
+    a[:, 0] = 1.0
+    for k in (64, 70, 74, 75):
+        res = solve_gpu(nx, ny, 2, "ring", "device", k, 0, init=a)
+        s = res["final"][0]
+        want = np.float32(2.0 ** (-2 * k)) if k <= 74 else np.float32(0.0)
+        assert s[1, k] == want and s[1, k + 1] == 0.0
+
+
+def test_zero_init_unit_boundary_subnormals_match_oracle():
+    a = np.zeros((4 + 2, 160), np.float32)
+    a[:, 0] = 1.0
+    a[2:4, 0] = 0.5
+    _check(160, 4, 1, "ring", "device", 90, norm_every=10, init=a)
+
+
+def test_constant_field_fixed_and_zero_norm():
+    a = np.full((34, 64), 0.7, np.float32)
+    res = solve_gpu(64, 32, 4, "ring", "device", 5, 1, init=a)
+    for s in res["final"]:
+        assert np.array_equal(bits(s), bits(np.full_like(s, 0.7)))
+    assert not res["norms"].any()
+
+
+# --------------------------------------------------------------------------- full size
+def test_full_size_16384_single_gpu_bench_configuration():
+    """BASELINE.json configs[2]/[3] at P = 1 (16384^2 fp32, 1 GiB per slab), in the launch
+    configuration bench.py times (device mode, ring, CUDA graph, default geometry): the whole
+    grid bit-exact vs the oracle after 6 iterations, norms within 1e-5."""
+    _check(16384, 16384, 1, "ring", "device", 6, norm_every=3)
+
+
+def test_full_size_host_mode():
+    _check(16384, 16384, 1, "ring", "host", 2, norm_every=1)
