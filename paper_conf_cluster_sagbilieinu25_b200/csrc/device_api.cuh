@@ -42,7 +42,9 @@ __device__ __forceinline__ bool wait_ge(const uint64_t* flag, uint64_t v, unsign
   unsigned long long t0 = globaltimer();
   unsigned ns = 32;
   while (ld_acquire_sys(flag) < v) {
-    if (globaltimer() - t0 > timeout_ns) {
+    // give up at the timeout, or at once if an earlier wait already timed out (so a broken
+    // peer costs one timeout, not one per pending wait)
+    if (globaltimer() - t0 > timeout_ns || *(volatile unsigned int*)err) {
       atomicOr(err, 1u);
       return false;
     }

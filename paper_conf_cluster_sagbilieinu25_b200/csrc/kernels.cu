@@ -28,6 +28,8 @@
 #include "device_api.cuh"
 #include "uc_internal.h"
 
+extern "C" __global__ void uc_fill_f32(float* dst, unsigned long long n, float value);
+
 namespace uc {
 using namespace dev;
 
@@ -129,7 +131,7 @@ __device__ __forceinline__ void march(const float* __restrict__ src, float* __re
         const float4 dn = nb[i];
         const float4 o = row_update(up, cur, dn, ec, lane, x4, nx4);
         if (valid) __stcs(reinterpret_cast<float4*>(dst + (size_t)(y + i) * pitch) + x4, o);
-        if (NORM) acc_sq(acc, o, cur);
+        if (NORM && valid) acc_sq(acc, o, cur);  // lanes past the row end hold garbage
         up = cur;
         cur = dn;
         ec = ne[i];
@@ -156,7 +158,7 @@ __device__ __forceinline__ void boundary_row(const JacobiParams& p, const float*
   if (threadIdx.x == 0) {
     // halo rows of A_k (slab k&1) must hold the neighbours' A_k rows: wait for flag >= k
     if (put_top) wait_ge(p.my_flags + (size_t)s * kFlagStride, k, p.timeout_ns, p.err);
-    if (put_bot) wait_ge(p.my_flags + (size_t)(p.strips + s) * kFlagStride, k, p.timeout_ns, p.err);
+    if (put_bot) wait_ge(p.my_flags + (size_t)(p.flag_half + s) * kFlagStride, k, p.timeout_ns, p.err);
   }
   __syncthreads();
   const bool valid = x4 < p.nx4;
@@ -173,12 +175,12 @@ __device__ __forceinline__ void boundary_row(const JacobiParams& p, const float*
     if (put_top) reinterpret_cast<float4*>(p.top_slab[np] + (size_t)(p.n + 1) * pitch)[x4] = o;
     if (put_bot) reinterpret_cast<float4*>(p.bot_slab[np])[x4] = o;
   }
-  if (NORM) acc_sq(acc, o, cur);
+  if (NORM && valid) acc_sq(acc, o, cur);
   if (put_top || put_bot) {
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence_system();
-      if (put_top) st_release_sys(p.top_flags + (size_t)(p.strips + s) * kFlagStride, k + 1);  // top's from_bottom[s]
+      if (put_top) st_release_sys(p.top_flags + (size_t)(p.flag_half + s) * kFlagStride, k + 1);  // top's from_bottom[s]
       if (put_bot) st_release_sys(p.bot_flags + (size_t)s * kFlagStride, k + 1);               // bottom's from_top[s]
     }
   }
@@ -465,6 +467,21 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
   allreduce_oneshot_kernel<<<1, 256, 0, s>>>(send, recv, count, dtype, rank, size, sp, fp, my_flags,
                                              (const char*)my_slots, epoch, slot_bytes, timeout_ns, err);
   UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+// Load every kernel of this module now.  With CUDA lazy loading a kernel's first launch may
+// need a context-wide synchronisation; a rank whose kernel spins on a peer's kernel (device
+// mode) must never depend on such a load happening concurrently.
+int preload_kernels() {
+  const void* fns[] = {(const void*)jacobi_iter_kernel, (const void*)norm_finish_kernel,
+                       (const void*)init_field_kernel,  (const void*)put_signal_kernel,
+                       (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
+                       (const void*)uc_fill_f32};
+  for (const void* f : fns) {
+    cudaFuncAttributes a;
+    UC_CUDA(cudaFuncGetAttributes(&a, f));
+  }
   return UC_OK;
 }
 

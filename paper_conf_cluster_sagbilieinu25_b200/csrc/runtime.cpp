@@ -94,6 +94,7 @@ int uc_env_init(int world_rank, int world_size, int device, uc_allgather_fn ag, 
     if (device < 0 || device >= ndev) return fail(UC_ERR_ARG, "device %d not in [0, %d)", device, ndev);
     UC_CUDA(cudaSetDevice(device));
     UC_CUDA(cudaFree(nullptr));  // create the primary context now
+    UC_TRY(preload_kernels());   // no lazy module loads once ranks spin on each other
   }
   uc_env* e = new uc_env;
   e->rank = world_rank;
@@ -243,7 +244,7 @@ int uc_mem_alloc_symmetric(uc_comm* c, size_t bytes, uc_mem** out) {
     return fail(UC_ERR_OOM, "cudaMalloc(%zu): %s", bytes, cudaGetErrorString(e));
   }
   UC_CUDA(cudaMemset(p, 0, bytes));
-  UC_CUDA(cudaDeviceSynchronize());
+  UC_CUDA(cudaStreamSynchronize(nullptr));
   IpcRecord rec{};
   rec.raw = (uint64_t)(uintptr_t)p;
   bool need_ipc = false;
@@ -318,7 +319,7 @@ int uc_mem_free_symmetric(uc_mem* m) {
   if (!m) return fail(UC_ERR_ARG, "mem is NULL");
   uc_comm* c = m->comm;
   UC_CUDA(cudaSetDevice(c->env->device));
-  UC_CUDA(cudaDeviceSynchronize());
+  UC_CUDA(cudaStreamSynchronize(nullptr));
   UC_TRY(uc_comm_barrier(c, nullptr));  // nobody still writes into our buffer
   for (int q = 0; q < c->size; ++q)
     if (m->ipc_opened[q]) cudaIpcCloseMemHandle(m->ptrs[q]);
@@ -351,7 +352,7 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
   if (e == cudaSuccess) e = cudaMemset(k->err, 0, sizeof(unsigned int));
   if (e == cudaSuccess) e = cudaMalloc(&k->put_counter, sizeof(unsigned int));
   if (e == cudaSuccess) e = cudaMemset(k->put_counter, 0, sizeof(unsigned int));
-  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
   if (e != cudaSuccess) return cleanup(fail(UC_ERR_CUDA, "coordinator state: %s", cudaGetErrorString(e)));
   if (mode == UC_MODE_HOST) {
     ncclUniqueId id{};

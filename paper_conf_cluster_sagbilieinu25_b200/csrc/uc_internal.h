@@ -61,6 +61,7 @@ struct JacobiParams {
   int nx, n;               // columns, owned rows
   int nx4;                 // nx / 4
   int strips, chunks;      // grid = strips * chunks blocks
+  int flag_half;           // from_bottom flags start at index flag_half (= max strips)
   int has_top, has_bot;
   int device_mode;         // 1: fused waits + puts + in-kernel cross-rank norm
   int norm_every;          // <= 0: never
@@ -86,6 +87,7 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
                              const void* my_slots, uint64_t epoch, size_t slot_bytes,
                              unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 int jacobi_occupancy(int block, int* blocks_per_sm);
+int preload_kernels();
 const void* builtin_kernel(const char* name);
 
 }  // namespace uc
@@ -156,7 +158,8 @@ struct uc_jacobi {
   uc_mem* slabs = nullptr;       // symmetric: 2 * (n+2) * nx floats
   uc_mem* ctrl = nullptr;        // symmetric: flags + norm slots
   size_t slab_elems = 0;
-  int strips = 0;
+  int strips = 0;               // current column strips (launch geometry)
+  int max_strips = 0;           // flag capacity per side = ceil(nx/4 / 32)
   // local device state
   unsigned long long* k_dev = nullptr;
   unsigned int* done = nullptr;
@@ -164,6 +167,7 @@ struct uc_jacobi {
   double* rank_sum = nullptr;
   double* norm_hist = nullptr;
   int norm_cap = 4096;
+  cudaStream_t aux = nullptr;    // private non-blocking stream (init, synchronous copies)
   int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
   int partials_cap = 0;
   std::vector<JacobiGraph> graphs;

@@ -29,7 +29,7 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
         comm = U.Comm(env, top, bot)
         stream = torch.cuda.Stream()
         coord = U.Coord(comm, MODES[mode], stream.cuda_stream)
-        coord.set_timeout(30.0)
+        coord.set_timeout(5.0)
         J = U.Jacobi(comm, nx, ny, seed, zero_init)
         try:
             if block_x or blocks_per_sm:
@@ -37,6 +37,7 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
             slab0 = J.copy_out()
             if init is not None:
                 J.copy_in(gen.rank_slab(init, rank, P))
+            comm.barrier()
             if stepwise:
                 norms = []
                 for i in range(iters):

@@ -57,6 +57,18 @@ def test_ragged_shapes_single_rank(nx, ny, iters, topology):
     _check(nx, ny, 1, topology, "device", iters, norm_every=4)
 
 
+@pytest.mark.parametrize("nx", [1028, 4, 36])
+def test_ragged_random_boundaries(nx):
+    """Random values everywhere, including both fixed columns, with a ragged last strip: lanes
+    past the row end must neither write nor enter the norm."""
+    ny = 12
+    rng = np.random.default_rng(nx)
+    init = rng.random((ny + 2, nx), dtype=np.float32)
+    init[0], init[-1] = init[ny], init[1]  # ring halos
+    _check(nx, ny, 1, "ring", "device", 7, norm_every=2, init=init)
+    _check(nx, ny, 2, "dirichlet", "device", 7, norm_every=2, init=init)
+
+
 @pytest.mark.parametrize("P", [2, 3, 4, 8])
 @pytest.mark.parametrize("topology", ["ring", "dirichlet"])
 def test_partition_invariance_device_mode(P, topology):

@@ -30,7 +30,7 @@ def _setup(rank, P, ag, mode):
     comm = U.Comm(env, *U.ring_neighbours(rank, P))
     stream = torch.cuda.Stream()
     coord = U.Coord(comm, mode, stream.cuda_stream)
-    coord.set_timeout(20.0)
+    coord.set_timeout(5.0)
     return U, env, comm, stream, coord
 
 
