@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
     ap.add_argument("--cpu-sample-iters", type=int, default=3)
+    ap.add_argument("--variant", type=int, default=-1, help="0 register march, 1 TMA-staged (-1: library default)")
+    ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--block-x", type=int, default=0)
     ap.add_argument("--blocks-per-sm", type=int, default=0)
     return ap.parse_args()
@@ -182,8 +184,8 @@ def run_ours(a):
     stream = torch.cuda.Stream()
     coord = U.Coord(comm, mode, stream.cuda_stream)
     J = U.Jacobi(comm, nx, ny)
-    if a.block_x or a.blocks_per_sm:
-        J.set_launch(a.block_x, a.blocks_per_sm)
+    if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages:
+        J.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages)
     n = J.n
     launch_info = J.launch_info()
     use_graph = not a.no_graph

@@ -10,7 +10,8 @@ import ctypes as C
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libuniconn_b200.so")
+# UC_LIB_PATH selects an A/B build of the same CUDA sources (build.py --define ... --out ...).
+LIB_PATH = os.environ.get("UC_LIB_PATH") or os.path.join(_PKG, "libuniconn_b200.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: run `python -m paper_conf_cluster_sagbilieinu25_b200.build` "
@@ -65,8 +66,8 @@ _SIGS = {
     "uc_jacobi_copy_out_async": (i32, [vp, vp, vp]),
     "uc_jacobi_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32), P(i64)]),
     "uc_jacobi_destroy": (i32, [vp]),
-    "uc_jacobi_set_launch": (i32, [vp, i32, i32]),
-    "uc_jacobi_launch_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32)]),
+    "uc_jacobi_set_launch": (i32, [vp, i32, i32, i32, i32]),
+    "uc_jacobi_launch_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32), P(i32), P(i32)]),
     "uc_last_error": (C.c_char_p, []),
     "uc_status_string": (C.c_char_p, [i32]),
     "uc_version": (i32, []),

@@ -51,12 +51,17 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """Build the library.  `defines` (e.g. ["UC_KR=8"]) and `out` produce A/B builds of the same
+    sources (compile-time tuning knobs in csrc/kernels.cu), loaded with UC_LIB_PATH=<out>."""
+    target = out or LIB
+    if not force and not defines and out is None and not _stale():
         return LIB
     nd = nccl_dir()
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc(), *ARCH, *NVCC_FLAGS, "-shared", "-I", INCLUDE, "-I", CSRC, "-I", os.path.join(nd, "include"),
+    os.makedirs(os.path.dirname(os.path.abspath(target)), exist_ok=True)
+    tmp = target + f".tmp{os.getpid()}"
+    cmd = [nvcc(), *ARCH, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-shared", "-I", INCLUDE, "-I", CSRC,
+           "-I", os.path.join(nd, "include"),
            *sources(), "-o", tmp, "-L", os.path.join(nd, "lib"), "-l:libnccl.so.2",
            "-Xlinker", "-rpath=" + os.path.join(nd, "lib")]
     res = subprocess.run(cmd, capture_output=True, text=True)
@@ -68,9 +73,16 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError(f"nvcc failed (see {log})")
     if verbose:
         sys.stderr.write(res.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    import argparse
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--force", action="store_true")
+    ap.add_argument("-v", action="store_true")
+    ap.add_argument("--define", action="append", default=[])
+    ap.add_argument("--out", default=None)
+    a = ap.parse_args()
+    print(build(force=a.force, verbose=a.v, defines=a.define, out=a.out))

@@ -34,7 +34,32 @@ namespace uc {
 using namespace dev;
 
 constexpr unsigned kFull = 0xffffffffu;
-constexpr int kR = 4;          // rows per prefetch batch
+// Compile-time tuning knobs (A/B builds via build.py --define; defaults are the product build).
+#ifndef UC_KR
+#define UC_KR 4
+#endif
+#ifndef UC_STORE_CS
+#define UC_STORE_CS 1
+#endif
+#ifndef UC_MINBLOCKS
+#define UC_MINBLOCKS 1
+#endif
+constexpr int kR = UC_KR;      // rows per prefetch batch
+#ifndef UC_STAGE_PAD
+#define UC_STAGE_PAD 4
+#endif
+constexpr int kPad = UC_STAGE_PAD;  // staged ring: halo floats copied on each side of a strip
+#ifndef UC_L2_EVICT_FIRST
+#define UC_L2_EVICT_FIRST 1
+#endif
+
+__device__ __forceinline__ void st4(float* p, float4 v) {
+#if UC_STORE_CS
+  __stcs(reinterpret_cast<float4*>(p), v);  // streaming: the result is read next iteration from HBM
+#else
+  *reinterpret_cast<float4*>(p) = v;
+#endif
+}
 constexpr int kMaxBlock = 256; // threads per block (upper bound)
 
 // ------------------------------------------------------------------------------ stencil math
@@ -130,7 +155,7 @@ __device__ __forceinline__ void march(const float* __restrict__ src, float* __re
       if (y + i <= y1) {
         const float4 dn = nb[i];
         const float4 o = row_update(up, cur, dn, ec, lane, x4, nx4);
-        if (valid) __stcs(reinterpret_cast<float4*>(dst + (size_t)(y + i) * pitch) + x4, o);
+        if (valid) st4(dst + (size_t)(y + i) * pitch + 4 * (size_t)x4, o);
         if (NORM && valid) acc_sq(acc, o, cur);  // lanes past the row end hold garbage
         up = cur;
         cur = dn;
@@ -239,16 +264,89 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
   }
 }
 
-// ------------------------------------------------------------------------------ the kernel
+// ------------------------------------------------------------------------------ staged y-march
+// Variant 1: the rows of this block's strip are staged into a shared-memory ring by the TMA
+// engine (cp.async.bulk, one copy per row of 4*nc+8 floats incl. a 4-float halo on each side),
+// issued by a dedicated producer warp ahead of the consumers; mbarriers carry "full" (bytes
+// landed) and "empty" (all consumer warps copied the row out) per stage.  Up to NS-1 rows per
+// block are in flight without costing registers, which is what keeps HBM busy.
+// Ring layout: stage i = floats [i*ST, (i+1)*ST), ST = 4*nc + 8; column x0 - 4 sits at 0.
 template <bool NORM>
-__device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t k) {
+__device__ __forceinline__ void march_staged(const JacobiParams& p, const float* src, float* dst, int s,
+                                             int x4, bool valid, int y0, int y1, double& acc, float* ring,
+                                             uint64_t* full, uint64_t* empty) {
+  const int nc = p.consumers, NS = p.stages;
+  const int ST = 4 * nc + 2 * kPad;
+  const int lane = threadIdx.x & 31;
+  const size_t pitch = (size_t)p.nx;
+  const int rows = y1 - y0 + 3;  // y0-1 .. y1+1
+  if ((int)threadIdx.x >= nc) {
+    // ---- producer warp (one lane issues every copy)
+    if (lane == 0) {
+      const int x0 = s * 4 * nc;  // first column of the strip
+      const int left = x0 >= kPad ? x0 - kPad : 0;
+      const int right = min(x0 + 4 * nc + kPad, p.nx);
+      const unsigned bytes = (unsigned)(right - left) * 4u;
+      const int off = left - (x0 - kPad);  // kPad for the first strip, else 0
+#if UC_L2_EVICT_FIRST
+      const uint64_t pol = policy_evict_first();
+#else
+      const uint64_t pol = policy_evict_normal();
+#endif
+      for (int i = 0; i < rows; ++i) {
+        const int st = i % NS;
+        if (i >= NS) mbar_wait(empty + st, (unsigned)((i / NS) - 1) & 1u);
+        mbar_arrive_expect_tx(full + st, bytes);
+        bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(y0 - 1 + i) * pitch + left, bytes, full + st, pol);
+      }
+    }
+    return;
+  }
+  // ---- consumer warps: copy the new row out of the ring, release the stage, compute
+  const int t = threadIdx.x;
+  float4 up = make_float4(0.f, 0.f, 0.f, 0.f), cur = up;
+  float ec = 0.f;
+  for (int i = 0; i < rows; ++i) {
+    const int st = i % NS;
+    mbar_wait(full + st, (unsigned)(i / NS) & 1u);
+    const float* row = ring + (size_t)st * ST + kPad + 4 * t;
+    const float4 v = *reinterpret_cast<const float4*>(row);
+    float e = 0.f;
+    if (lane == 0) e = row[-1];
+    else if (lane == 31) e = row[4];
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty + st);
+    if (i == 0) {
+      up = v;
+    } else if (i == 1) {
+      cur = v;
+      ec = e;
+    } else {
+      const int y = y0 + i - 2;
+      const float4 o = row_update(up, cur, v, ec, lane, x4, p.nx4);
+      if (valid) st4(dst + (size_t)y * pitch + 4 * (size_t)x4, o);
+      if (NORM && valid) acc_sq(acc, o, cur);
+      up = cur;
+      cur = v;
+      ec = e;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------ the kernel
+template <int VARIANT, bool NORM>
+__device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t k, float* ring, uint64_t* full,
+                                                 uint64_t* empty) {
   const int par = (int)(k & 1);
   const float* src = p.slab[par];
   float* dst = p.slab[par ^ 1];
   const int s = blockIdx.x % p.strips;
   const int q = blockIdx.x / p.strips;
   const int lane = threadIdx.x & 31;
-  const int x4 = s * blockDim.x + threadIdx.x;
+  const int nc = VARIANT == 0 ? (int)blockDim.x : p.consumers;
+  // the producer warp of variant 1 owns no column
+  const int x4 = (int)threadIdx.x < nc ? s * nc + (int)threadIdx.x : 0x3fffffff;
+  const bool valid = x4 < p.nx4;
   const int lo = 1 + (int)(((long long)q * p.n) / p.chunks);
   const int hi = (int)(((long long)(q + 1) * p.n) / p.chunks);
   double acc = 0.0;
@@ -259,21 +357,42 @@ __device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t
     if (a < 2) a = 2;
     if (b > p.n - 1) b = p.n - 1;
   }
-  if (a <= b) march<NORM>(src, dst, p.nx, p.nx4, x4, lane, a, b, acc);
+  if (a <= b) {
+    if (VARIANT == 0) march<NORM>(src, dst, p.nx, p.nx4, x4, lane, a, b, acc);
+    else march_staged<NORM>(p, src, dst, s, x4, valid, a, b, acc, ring, full, empty);
+  }
   return acc;
 }
 
-__global__ void __launch_bounds__(kMaxBlock) jacobi_iter_kernel(const JacobiParams p) {
-  __shared__ double smem[kMaxBlock / 32];
+template <int VARIANT>
+__global__ void __launch_bounds__(kMaxBlock + 32, UC_MINBLOCKS) jacobi_iter_kernel(const JacobiParams p) {
+  __shared__ double smem[32];
   __shared__ int s_last;
+  extern __shared__ __align__(128) unsigned char dyn[];
+  float* ring = nullptr;
+  uint64_t *full = nullptr, *empty = nullptr;
+  if (VARIANT == 1) {
+    const int NS = p.stages;
+    full = reinterpret_cast<uint64_t*>(dyn);
+    empty = full + NS;
+    ring = reinterpret_cast<float*>(dyn + ((16 * NS + 127) / 128) * 128);  // after 2*NS mbarriers
+    if (threadIdx.x == 0) {
+      for (int i = 0; i < NS; ++i) {
+        mbar_init(full + i, 1);                   // the producer's arrive.expect_tx
+        mbar_init(empty + i, p.consumers / 32);   // one arrive per consumer warp
+      }
+      fence_mbar_init();
+    }
+    __syncthreads();
+  }
   const uint64_t k = p.k_dev[0];
   const bool do_norm = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
   if (do_norm) {
-    const double acc = iteration_body<true>(p, k);
+    const double acc = iteration_body<VARIANT, true>(p, k, ring, full, empty);
     const double t = block_sum(acc, smem);
     if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
   } else {
-    iteration_body<false>(p, k);
+    iteration_body<VARIANT, false>(p, k, ring, full, empty);
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -412,8 +531,15 @@ __global__ void allreduce_oneshot_kernel(const void* send, void* recv, size_t co
 }
 
 // ------------------------------------------------------------------------------ launchers
+size_t staged_smem_bytes(int consumers, int stages) {
+  return (size_t)((16 * stages + 127) / 128) * 128 + (size_t)stages * (4 * consumers + 2 * kPad) * sizeof(float);
+}
+
 int launch_jacobi_iteration(const JacobiParams& p, int block, cudaStream_t s) {
-  jacobi_iter_kernel<<<p.strips * p.chunks, block, 0, s>>>(p);
+  if (p.variant == 1)
+    jacobi_iter_kernel<1><<<p.strips * p.chunks, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p);
+  else
+    jacobi_iter_kernel<0><<<p.strips * p.chunks, block, 0, s>>>(p);
   UC_CUDA(cudaGetLastError());
   return UC_OK;
 }
@@ -474,7 +600,9 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
 // need a context-wide synchronisation; a rank whose kernel spins on a peer's kernel (device
 // mode) must never depend on such a load happening concurrently.
 int preload_kernels() {
-  const void* fns[] = {(const void*)jacobi_iter_kernel, (const void*)norm_finish_kernel,
+  UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  const void* fns[] = {(const void*)jacobi_iter_kernel<0>, (const void*)jacobi_iter_kernel<1>,
+                       (const void*)norm_finish_kernel,
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
                        (const void*)uc_fill_f32};
@@ -485,8 +613,11 @@ int preload_kernels() {
   return UC_OK;
 }
 
-int jacobi_occupancy(int block, int* blocks_per_sm) {
-  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel, block, 0));
+int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm) {
+  if (variant == 1)
+    UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<1>, block, smem));
+  else
+    UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<0>, block, 0));
   return UC_OK;
 }
 

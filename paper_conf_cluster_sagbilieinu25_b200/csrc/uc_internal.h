@@ -62,6 +62,9 @@ struct JacobiParams {
   int nx4;                 // nx / 4
   int strips, chunks;      // grid = strips * chunks blocks
   int flag_half;           // from_bottom flags start at index flag_half (= max strips)
+  int variant;             // 0: register y-march (LDG.128), 1: TMA-staged y-march (smem ring)
+  int consumers;           // variant 1: compute threads per block (a producer warp comes on top)
+  int stages;              // variant 1: ring depth (rows)
   int has_top, has_bot;
   int device_mode;         // 1: fused waits + puts + in-kernel cross-rank norm
   int norm_every;          // <= 0: never
@@ -70,6 +73,10 @@ struct JacobiParams {
 };
 
 constexpr int kFlagStride = 16;  // u64 per flag = 128 bytes, one flag per L2 line
+// Defaults from the round-1 sweep at 16384^2 (profiles/r1_sweep.txt): the TMA-staged march
+// with a 3-row ring reaches 6.36 TB/s vs 6.07 for the register march; deeper rings lose.
+constexpr int kDefaultVariant = 1;
+constexpr int kDefaultStages = 3;
 
 // Launch wrappers implemented in kernels.cu
 int launch_jacobi_iteration(const JacobiParams& p, int block, cudaStream_t s);
@@ -86,7 +93,8 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
                              void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
                              const void* my_slots, uint64_t epoch, size_t slot_bytes,
                              unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
-int jacobi_occupancy(int block, int* blocks_per_sm);
+int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm);
+size_t staged_smem_bytes(int consumers, int stages);
 int preload_kernels();
 const void* builtin_kernel(const char* name);
 
@@ -168,6 +176,7 @@ struct uc_jacobi {
   double* norm_hist = nullptr;
   int norm_cap = 4096;
   cudaStream_t aux = nullptr;    // private non-blocking stream (init, synchronous copies)
+  int variant = uc::kDefaultVariant, consumers = 0, stages = 0;
   int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
   int partials_cap = 0;
   std::vector<JacobiGraph> graphs;

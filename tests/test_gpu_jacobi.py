@@ -99,11 +99,66 @@ def test_graph_and_stepwise_agree():
     assert np.array_equal(a["norms"], c["norms"][[0, 7, 14, 21, 28]])
 
 
-@pytest.mark.parametrize("block_x,bps", [(32, 1), (64, 2), (128, 0), (256, 1)])
-def test_launch_geometries(block_x, bps):
-    """Different block widths / chunk counts change blocking, not results."""
-    res = _check(1024, 96, 1, "ring", "device", 9, norm_every=3, block_x=block_x, blocks_per_sm=bps)
-    assert res["launch"]["block"] == block_x
+@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("block_x,bps,stages", [(32, 1, 3), (64, 2, 4), (128, 0, 0), (256, 1, 16)])
+def test_launch_geometries(variant, block_x, bps, stages):
+    """Both kernel variants, different block widths / chunk counts / ring depths change the
+    blocking, not the results."""
+    res = _check(1024, 96, 1, "ring", "device", 9, norm_every=3, block_x=block_x, blocks_per_sm=bps,
+                 variant=variant, stages=stages)
+    assert res["launch"]["block"] == block_x + (32 if variant == 1 else 0)
+    assert res["launch"]["variant"] == variant
+
+
+STAGED = dict(variant=1)
+
+
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+@pytest.mark.parametrize("mode", ["device", "host"])
+def test_staged_variant_c1(topology, mode):
+    _check(256, 256, 1, topology, mode, 100, norm_every=10, **STAGED)
+
+
+@pytest.mark.parametrize("nx,ny,P", [(1028, 64, 1), (4, 2, 1), (2052, 33, 1), (520, 96, 4), (64, 3, 3),
+                                     (36, 16, 8)])
+def test_staged_variant_shapes(nx, ny, P):
+    for topology in ("ring", "dirichlet"):
+        _check(nx, ny, P, topology, "device", 13, norm_every=4, **STAGED)
+
+
+def test_switch_variant_mid_run():
+    """set_launch between runs (new strip layout, re-armed halo flags) keeps the iteration
+    bit-exact: 7 iterations of variant 0 (256-wide strips), 13 of variant 1 (64-wide strips)."""
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+    from vranks import run_ranks
+    nx, ny, P = 1028, 48, 2
+
+    def body(rank, P, ag):
+        env = U.Env(rank, P, 0, ag)
+        comm = U.Comm(env, *U.ring_neighbours(rank, P))
+        st = torch.cuda.Stream()
+        coord = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
+        coord.set_timeout(5.0)
+        J = U.Jacobi(comm, nx, ny)
+        n1 = J.run(coord, 7, 5)
+        coord.sync()
+        J.set_launch(1, 64, 0, 5)
+        n2 = J.run(coord, 13, 5)
+        coord.sync()
+        out = J.copy_out(coord)
+        comm.barrier()
+        J.destroy()
+        coord.destroy()
+        comm.destroy()
+        env.finalize()
+        return out, np.concatenate([n1, n2])
+
+    res = run_ranks(P, body)
+    _, want, want_norms = _oracle(nx, ny, "ring", 20, 5)
+    assert_slabs_equal_global([r[0] for r in res], want, P, "ring")
+    assert np.allclose(res[0][1], want_norms, rtol=NORM_RTOL, atol=0)
 
 
 # --------------------------------------------------------------------------- pinned examples
