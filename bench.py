@@ -43,7 +43,7 @@ NORM_EVERY = 100
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--mode", default="device", choices=["device", "host"])
@@ -53,6 +53,9 @@ def parse():
     ap.add_argument("--iters-per-step", type=int, default=ITERS_PER_STEP)
     ap.add_argument("--norm-every", type=int, default=NORM_EVERY)
     ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--same-device", action="store_true",
+                    help="TEST ONLY: put every rank on cuda:0 (exercises the multi-process path on a 1-GPU box; "
+                         "ranks time-slice the GPU, so the numbers are not a benchmark)")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
     ap.add_argument("--cpu-sample-iters", type=int, default=3)
     ap.add_argument("--variant", type=int, default=-1, help="0 register march, 1 TMA-staged (-1: library default)")
@@ -126,7 +129,7 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -172,6 +175,8 @@ def run_ours(a):
     import paper_conf_cluster_sagbilieinu25_b200 as U
 
     rank, world, local = dist_env()
+    if a.same_device:
+        local = 0
     if world != a.gpus:
         raise SystemExit(f"--gpus {a.gpus} but WORLD_SIZE={world}")
     dist = init_pg(rank, world)

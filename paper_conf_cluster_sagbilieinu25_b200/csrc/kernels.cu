@@ -474,6 +474,24 @@ __global__ void put_signal_kernel(const uint4* __restrict__ src, uint4* dst, siz
   }
 }
 
+// Device mode: the halo rows of the current iterate A_k are written by the neighbours during
+// THEIR iteration k-1, possibly after this rank finished its own; before the slab is read back
+// the stream waits for every per-strip flag >= k.
+__global__ void wait_halo_kernel(const uint64_t* my_flags, int strips, int flag_half, int has_top, int has_bot,
+                                 uint64_t k, unsigned long long timeout_ns, unsigned int* err) {
+  for (int s = threadIdx.x; s < strips; s += blockDim.x) {
+    if (has_top) wait_ge(my_flags + (size_t)s * kFlagStride, k, timeout_ns, err);
+    if (has_bot) wait_ge(my_flags + (size_t)(flag_half + s) * kFlagStride, k, timeout_ns, err);
+  }
+}
+
+int launch_wait_halo(const uint64_t* my_flags, int strips, int flag_half, int has_top, int has_bot, uint64_t k,
+                     unsigned long long timeout_ns, unsigned int* err, cudaStream_t s) {
+  wait_halo_kernel<<<1, 128, 0, s>>>(my_flags, strips, flag_half, has_top, has_bot, k, timeout_ns, err);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
 // Acknowledge (one-sided, device mode): the stream waits until the local signal >= val.
 __global__ void signal_wait_kernel(const uint64_t* sig, uint64_t val, unsigned long long timeout_ns,
                                    unsigned int* err) {
@@ -605,7 +623,7 @@ int preload_kernels() {
                        (const void*)norm_finish_kernel,
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
-                       (const void*)uc_fill_f32};
+                       (const void*)wait_halo_kernel,   (const void*)uc_fill_f32};
   for (const void* f : fns) {
     cudaFuncAttributes a;
     UC_CUDA(cudaFuncGetAttributes(&a, f));

@@ -94,6 +94,8 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
                              const void* my_slots, uint64_t epoch, size_t slot_bytes,
                              unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm);
+int launch_wait_halo(const uint64_t* my_flags, int strips, int flag_half, int has_top, int has_bot, uint64_t k,
+                     unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 size_t staged_smem_bytes(int consumers, int stages);
 int preload_kernels();
 const void* builtin_kernel(const char* name);
