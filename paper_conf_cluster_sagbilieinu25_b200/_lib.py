@@ -25,6 +25,7 @@ UC_OK, UC_ERR_ARG, UC_ERR_CUDA, UC_ERR_NCCL, UC_ERR_BOOTSTRAP, UC_ERR_TIMEOUT, U
 UC_MODE_HOST, UC_MODE_DEVICE, UC_MODE_PARTIAL = 0, 1, 2
 UC_F32, UC_F64, UC_U64 = 0, 1, 2
 UC_TOPO_NONE, UC_TOPO_RING, UC_TOPO_CHAIN = 0, 1, 2
+UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_P2P_HALO = 0, 1, 2
 UC_MAX_RANKS = 8
 
 ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p)
@@ -56,6 +57,7 @@ _SIGS = {
     "uc_put_signal": (i32, [vp, vp, vp, sz, sz, vp, sz, u64, i32]),
     "uc_signal_wait": (i32, [vp, vp, sz, sz, vp, sz, u64, i32]),
     "uc_allreduce_sum": (i32, [vp, vp, vp, sz, i32]),
+    "uc_p2p_bench": (i32, [vp, i32, vp, vp, sz, i32, i32, i32, i32, i32]),
     "uc_jacobi_create": (i32, [vp, i32, i32, u64, i32, P(vp)]),
     "uc_jacobi_step": (i32, [vp, vp, i32, vp]),
     "uc_jacobi_run": (i32, [vp, vp, i32, i32, vp, i32]),

@@ -19,6 +19,14 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
   return v;
 }
 
+__device__ __forceinline__ uint64_t ld_relaxed_sys_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+
 __device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
   asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -41,7 +49,9 @@ __device__ __forceinline__ bool wait_ge(const uint64_t* flag, uint64_t v, unsign
   if (ld_acquire_sys(flag) >= v) return true;
   unsigned long long t0 = globaltimer();
   unsigned ns = 32;
-  while (ld_acquire_sys(flag) < v) {
+  // poll with relaxed loads (no L1 invalidation per poll); the fence after the observing load
+  // turns it into an acquire pattern
+  while (ld_relaxed_sys_u64(flag) < v) {
     // give up at the timeout, or at once if an earlier wait already timed out (so a broken
     // peer costs one timeout, not one per pending wait)
     if (globaltimer() - t0 > timeout_ns || *(volatile unsigned int*)err) {
@@ -51,6 +61,7 @@ __device__ __forceinline__ bool wait_ge(const uint64_t* flag, uint64_t v, unsign
     __nanosleep(ns);
     if (ns < 256) ns <<= 1;
   }
+  fence_acq_rel_sys();
   return true;
 }
 

@@ -474,6 +474,142 @@ __global__ void put_signal_kernel(const uint4* __restrict__ src, uint4* dst, siz
   }
 }
 
+// ------------------------------------------------------------------------------ P2P microbenchmark
+// OSU-style device-initiated latency / bandwidth / halo patterns (§VI-B)
+// in ONE persistent cooperative kernel per rank: no launch per message, like the paper's
+// device-API benchmarks over NVSHMEM.  Blocks share each message; a grid barrier separates the
+// data stores from the single-thread release of the signal.
+__device__ __forceinline__ void grid_sync(unsigned int* count, unsigned int* gen, unsigned nblocks) {
+  __syncthreads();
+  if (nblocks == 1) return;
+  if (threadIdx.x == 0) {
+    const unsigned g = *(volatile unsigned int*)gen;
+    __threadfence();
+    if (atomicAdd(count, 1u) == nblocks - 1) {
+      *(volatile unsigned int*)count = 0;
+      __threadfence();
+      atomicAdd(gen, 1u);
+    } else {
+      while (*(volatile unsigned int*)gen == g) {
+      }
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+// copy this block's share of [0, n16) 16-byte words
+__device__ __forceinline__ void block_share_copy(uint4* dst, const uint4* src, size_t n16) {
+  const size_t stride = (size_t)gridDim.x * blockDim.x;
+  size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+  for (; i + 3 * stride < n16; i += 4 * stride) {
+    const uint4 a = src[i], b = src[i + stride], c = src[i + 2 * stride], d = src[i + 3 * stride];
+    dst[i] = a;
+    dst[i + stride] = b;
+    dst[i + 2 * stride] = c;
+    dst[i + 3 * stride] = d;
+  }
+  for (; i < n16; i += stride) dst[i] = src[i];
+}
+
+struct P2PArgs {
+  const uint4* src;     // local message (first `bytes` of the local buffer)
+  uint4* dst_peer;      // pingpong/window: peer buffer + bytes
+  uint4* dst_top;       // halo: top's buffer + 2*bytes (its "from bottom" zone)
+  uint4* dst_bot;       // halo: bottom's buffer + bytes (its "from top" zone)
+  uint64_t* sig_peer;   // peer's signal array
+  uint64_t* sig_top;
+  uint64_t* sig_bot;
+  uint64_t* sig_mine;
+  unsigned int* bar;    // [count, gen] grid barrier
+  size_t n16;
+  uint64_t base;        // first signal value of this call
+  int iters, window, pattern, role;
+  unsigned long long timeout_ns;
+  unsigned int* err;
+};
+
+__global__ void p2p_bench_kernel(P2PArgs a) {
+  const bool lead = blockIdx.x == 0 && threadIdx.x == 0;
+  for (int i = 0; i < a.iters; ++i) {
+    const uint64_t v = a.base + (uint64_t)i + 1;
+    if (a.pattern == UC_P2P_PINGPONG) {
+      if (a.role == 1) {  // responder: wait for the ping, then pong
+        if (lead) wait_ge(a.sig_mine, v, a.timeout_ns, a.err);
+        grid_sync(a.bar, a.bar + 1, gridDim.x);
+      }
+      block_share_copy(a.dst_peer, a.src, a.n16);
+      grid_sync(a.bar, a.bar + 1, gridDim.x);
+      if (lead) {
+        // st.release.sys is cumulative over the stores ordered before it by the barrier
+        st_release_sys(a.sig_peer, v);
+        if (a.role == 0) wait_ge(a.sig_mine, v, a.timeout_ns, a.err);
+      }
+      if (a.role == 0) grid_sync(a.bar, a.bar + 1, gridDim.x);
+    } else if (a.pattern == UC_P2P_WINDOW) {
+      const uint64_t w0 = a.base + (uint64_t)i * a.window;  // message w of round i signals w0+w+1
+      if (a.role == 0) {
+        for (int w = 0; w < a.window; ++w) {
+          block_share_copy(a.dst_peer, a.src, a.n16);
+          grid_sync(a.bar, a.bar + 1, gridDim.x);
+          if (lead) {
+            st_release_sys(a.sig_peer + 1, w0 + w + 1);
+          }
+        }
+        if (lead) wait_ge(a.sig_mine + 2, v, a.timeout_ns, a.err);  // ack of this window
+        grid_sync(a.bar, a.bar + 1, gridDim.x);
+      } else if (lead) {
+        wait_ge(a.sig_mine + 1, w0 + a.window, a.timeout_ns, a.err);
+        st_release_sys(a.sig_peer + 2, v);
+      }
+    } else {  // UC_P2P_HALO: put to top and bottom at once, wait for both neighbours
+      if (a.dst_top) block_share_copy(a.dst_top, a.src, a.n16);
+      if (a.dst_bot) block_share_copy(a.dst_bot, a.src, a.n16);
+      grid_sync(a.bar, a.bar + 1, gridDim.x);
+      if (lead) {
+        if (a.sig_top) st_release_sys(a.sig_top + 4, v);  // top's "from bottom"
+        if (a.sig_bot) st_release_sys(a.sig_bot + 3, v);  // bottom's "from top"
+        if (a.sig_top) wait_ge(a.sig_mine + 3, v, a.timeout_ns, a.err);
+        if (a.sig_bot) wait_ge(a.sig_mine + 4, v, a.timeout_ns, a.err);
+      }
+      grid_sync(a.bar, a.bar + 1, gridDim.x);
+    }
+  }
+}
+
+int launch_p2p_bench(const P2PLaunch& L, cudaStream_t s) {
+  P2PArgs a{};
+  a.src = (const uint4*)L.src;
+  a.dst_peer = (uint4*)L.dst_peer;
+  a.dst_top = (uint4*)L.dst_top;
+  a.dst_bot = (uint4*)L.dst_bot;
+  a.sig_peer = L.sig_peer;
+  a.sig_top = L.sig_top;
+  a.sig_bot = L.sig_bot;
+  a.sig_mine = L.sig_mine;
+  a.bar = L.bar;
+  a.n16 = L.bytes / 16;
+  a.base = L.base;
+  a.iters = L.iters;
+  a.window = L.window;
+  a.pattern = L.pattern;
+  a.role = L.role;
+  a.timeout_ns = L.timeout_ns;
+  a.err = L.err;
+  int per_sm = 0, dev = 0, sms = 0;
+  UC_CUDA(cudaGetDevice(&dev));
+  UC_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, p2p_bench_kernel, 512, 0));
+  int blocks = L.blocks > 0 ? L.blocks : (int)std::min<size_t>(std::max<size_t>(1, L.bytes / 65536), (size_t)sms);
+  // at most one block per SM: co-resident next to the other ranks' kernels (virtual ranks share
+  // the GPU).  A cooperative launch would guarantee co-residency but is serialised against other
+  // cooperative kernels on the device, which deadlocks partners that spin on each other.
+  blocks = std::min(blocks, std::min(per_sm, 1) * sms);
+  p2p_bench_kernel<<<blocks, 512, 0, s>>>(a);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
 // Device mode: the halo rows of the current iterate A_k are written by the neighbours during
 // THEIR iteration k-1, possibly after this rank finished its own; before the slab is read back
 // the stream waits for every per-strip flag >= k.
@@ -623,7 +759,8 @@ int preload_kernels() {
                        (const void*)norm_finish_kernel,
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
-                       (const void*)wait_halo_kernel,   (const void*)uc_fill_f32};
+                       (const void*)wait_halo_kernel,   (const void*)p2p_bench_kernel,
+                       (const void*)uc_fill_f32};
   for (const void* f : fns) {
     cudaFuncAttributes a;
     UC_CUDA(cudaFuncGetAttributes(&a, f));

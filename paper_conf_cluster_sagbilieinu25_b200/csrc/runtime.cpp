@@ -350,8 +350,10 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
   };
   cudaError_t e = cudaMalloc(&k->err, sizeof(unsigned int));
   if (e == cudaSuccess) e = cudaMemset(k->err, 0, sizeof(unsigned int));
-  if (e == cudaSuccess) e = cudaMalloc(&k->put_counter, sizeof(unsigned int));
-  if (e == cudaSuccess) e = cudaMemset(k->put_counter, 0, sizeof(unsigned int));
+  // [0] put_signal block ticket, [1..2] p2p benchmark grid barrier (count, generation)
+  if (e == cudaSuccess) e = cudaMalloc(&k->put_counter, 4 * sizeof(unsigned int));
+  if (e == cudaSuccess) e = cudaMemset(k->put_counter, 0, 4 * sizeof(unsigned int));
+  k->p2p_bar = k->put_counter + 1;
   if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
   if (e != cudaSuccess) return cleanup(fail(UC_ERR_CUDA, "coordinator state: %s", cudaGetErrorString(e)));
   if (mode == UC_MODE_HOST) {
@@ -514,6 +516,59 @@ int uc_signal_wait(uc_coord* k, uc_mem* dst, size_t dst_off, size_t bytes, uc_me
 }
 
 // ============================================================================ AllReduce
+int uc_p2p_bench(uc_coord* k, int pattern, uc_mem* buf, uc_mem* sig, size_t bytes, int iters, int window, int peer,
+                 int role, int blocks) {
+  if (!k || !buf || !sig) return fail(UC_ERR_ARG, "NULL argument");
+  if (k->mode != UC_MODE_DEVICE) return fail(UC_ERR_UNSUPPORTED, "uc_p2p_bench runs device-initiated patterns only");
+  if (pattern < UC_P2P_PINGPONG || pattern > UC_P2P_HALO) return fail(UC_ERR_ARG, "unknown pattern %d", pattern);
+  if (bytes == 0 || bytes % 16) return fail(UC_ERR_ARG, "bytes must be a positive multiple of 16");
+  if (iters < 1 || (pattern == UC_P2P_WINDOW && window < 1)) return fail(UC_ERR_ARG, "iters/window must be >= 1");
+  if (sig->bytes < 8 * sizeof(uint64_t)) return fail(UC_ERR_ARG, "sig needs >= 8 u64");
+  const size_t need = (pattern == UC_P2P_HALO ? 3 : 2) * bytes;
+  if (buf->bytes < need) return fail(UC_ERR_ARG, "buf has %zu bytes, pattern needs %zu", buf->bytes, need);
+  uc_comm* c = k->comm;
+  UC_CUDA(cudaSetDevice(c->env->device));
+  P2PLaunch L{};
+  L.src = buf->local;
+  L.sig_mine = (uint64_t*)sig->local;
+  if (pattern == UC_P2P_HALO) {
+    if (c->top >= 0) {
+      L.dst_top = (char*)uc_mem_ptr(buf, c->top) + 2 * bytes;
+      L.sig_top = (uint64_t*)uc_mem_ptr(sig, c->top);
+    }
+    if (c->bottom >= 0) {
+      L.dst_bot = (char*)uc_mem_ptr(buf, c->bottom) + bytes;
+      L.sig_bot = (uint64_t*)uc_mem_ptr(sig, c->bottom);
+    }
+    if ((c->top >= 0 && (!L.dst_top || !L.sig_top)) || (c->bottom >= 0 && (!L.dst_bot || !L.sig_bot)))
+      return fail(UC_ERR_UNSUPPORTED, "a neighbour is not peer-addressable");
+  } else {
+    if (peer < 0 || peer >= c->size) return fail(UC_ERR_ARG, "peer %d out of range", peer);
+    if (role != 0 && role != 1) return fail(UC_ERR_ARG, "role must be 0 or 1");
+    L.dst_peer = (char*)uc_mem_ptr(buf, peer);
+    L.sig_peer = (uint64_t*)uc_mem_ptr(sig, peer);
+    if (!L.dst_peer || !L.sig_peer) return fail(UC_ERR_UNSUPPORTED, "rank %d not peer-addressable", peer);
+    L.dst_peer = (char*)L.dst_peer + bytes;
+  }
+  L.bar = k->p2p_bar;
+  L.bytes = bytes;
+  // signal slots are disjoint per pattern (0: ping-pong, 1-2: window, 3-4: halo) and each
+  // (pattern, peer) pair keeps its own monotone base, so partners only need to agree on the
+  // calls they make together
+  uint64_t& epoch = k->p2p_epoch[pattern][pattern == UC_P2P_HALO ? 0 : peer];
+  L.base = epoch;
+  L.iters = iters;
+  L.window = pattern == UC_P2P_WINDOW ? window : 1;
+  L.pattern = pattern;
+  L.role = role;
+  L.blocks = blocks;
+  L.timeout_ns = k->timeout_ns;
+  L.err = k->err;
+  // every signal value of this call lies in (base, base + iters*window]; both partners advance alike
+  epoch += (uint64_t)iters * (uint64_t)L.window + 1;
+  return launch_p2p_bench(L, k->stream);
+}
+
 int uc_allreduce_sum(uc_coord* k, const void* send, void* recv, size_t count, uc_dtype dt) {
   if (!k || !send || !recv) return fail(UC_ERR_ARG, "NULL argument");
   if (dt != UC_F32 && dt != UC_F64 && dt != UC_U64) return fail(UC_ERR_ARG, "unknown dtype %d", (int)dt);

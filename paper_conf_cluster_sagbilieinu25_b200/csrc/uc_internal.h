@@ -94,6 +94,18 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
                              const void* my_slots, uint64_t epoch, size_t slot_bytes,
                              unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm);
+struct P2PLaunch {
+  const void* src;
+  void *dst_peer, *dst_top, *dst_bot;
+  uint64_t *sig_peer, *sig_top, *sig_bot, *sig_mine;
+  unsigned int* bar;
+  size_t bytes;
+  uint64_t base;
+  int iters, window, pattern, role, blocks;
+  unsigned long long timeout_ns;
+  unsigned int* err;
+};
+int launch_p2p_bench(const P2PLaunch& L, cudaStream_t s);
 int launch_wait_halo(const uint64_t* my_flags, int strips, int flag_half, int has_top, int has_bot, uint64_t k,
                      unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 size_t staged_smem_bytes(int consumers, int stages);
@@ -150,6 +162,8 @@ struct uc_coord {
   uc_mem* ar_scratch = nullptr;        // device-mode allreduce slots [2][P][slot_bytes] + flags
   size_t ar_slot_bytes = 32768;
   uint64_t ar_epoch = 0;
+  uint64_t p2p_epoch[3][UC_MAX_RANKS] = {};  // signal base of the next uc_p2p_bench call, per (pattern, peer)
+  unsigned int* p2p_bar = nullptr;     // grid barrier [count, gen] of the p2p kernel
   int live_jacobi_users = 0;
 };
 

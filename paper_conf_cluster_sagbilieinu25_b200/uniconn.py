@@ -19,7 +19,8 @@ from typing import Callable, Optional
 import numpy as np
 
 from ._lib import (ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
-                   UC_TOPO_CHAIN, UC_TOPO_NONE, UC_TOPO_RING, UC_U64, UCError, check, lib)
+                   UC_P2P_HALO, UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_TOPO_CHAIN, UC_TOPO_NONE, UC_TOPO_RING, UC_U64,
+                   UCError, check, lib)
 
 AllgatherImpl = Callable[[bytes, int], bytes]  # (my bytes, bytes_per_rank) -> size*bytes_per_rank bytes
 
@@ -177,6 +178,11 @@ class Coord:
                     sig_val: int, peer: int):
         check(lib.uc_signal_wait(self.h, dst.h if dst else None, dst_off, nbytes, sig.h if sig else None, sig_idx,
                                  sig_val, peer), "uc_signal_wait")
+
+    def p2p_bench(self, pattern: int, buf: SymMem, sig: SymMem, nbytes: int, iters: int, window: int = 1,
+                  peer: int = 0, role: int = 0, blocks: int = 0):
+        check(lib.uc_p2p_bench(self.h, pattern, buf.h, sig.h, nbytes, iters, window, peer, role, blocks),
+              "uc_p2p_bench")
 
     def allreduce_sum(self, send: int, recv: int, count: int, dtype: int):
         check(lib.uc_allreduce_sum(self.h, C.c_void_p(send), C.c_void_p(recv), count, dtype), "uc_allreduce_sum")

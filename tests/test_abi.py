@@ -41,6 +41,14 @@ def test_binary_is_sm100a():
     assert "sm_100a" in out
 
 
+def test_enum_constants_match_header():
+    hdr = open(os.path.join(ROOT, "include", "uniconn.h")).read()
+    for name, val in re.findall(r"\b(UC_[A-Z0-9_]+)\s*=\s*(\d+)", hdr):
+        assert getattr(U, name, None) == int(val) or getattr(U._lib, name) == int(val), name
+    for name in ("UC_P2P_PINGPONG", "UC_P2P_WINDOW", "UC_P2P_HALO", "UC_MODE_DEVICE", "UC_TOPO_RING", "UC_F64"):
+        assert hasattr(U, name), name
+
+
 def test_status_strings_and_errors():
     assert U.lib.uc_status_string(0) == b"UC_OK"
     assert U.lib.uc_status_string(5) == b"UC_ERR_TIMEOUT"

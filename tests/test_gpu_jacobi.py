@@ -214,3 +214,20 @@ def test_full_size_16384_single_gpu_bench_configuration():
 
 def test_full_size_host_mode():
     _check(16384, 16384, 1, "ring", "host", 2, norm_every=1)
+
+
+def test_config1_4096_2ranks_1000_iterations():
+    """BASELINE.json configs[1]: 4096 x 4096, 1000 iterations, row-split over 2 ranks, device
+    put-signal (virtual ranks on one GPU), norm every 100: whole grid bit-exact."""
+    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100)
+
+
+def test_config2_strong_16384_over_8_ranks():
+    """BASELINE.json configs[2] at P = 8 (2048 rows per rank), norm allreduce every iteration
+    here (every 100 in the benchmark): whole grid bit-exact after 4 iterations."""
+    _check(16384, 16384, 8, "ring", "device", 4, norm_every=2)
+
+
+def test_config3_weak_16384_per_rank_2_ranks():
+    """BASELINE.json configs[3] at P = 2: 16384 x 32768 global, 16384 x 16384 per rank."""
+    _check(16384, 32768, 2, "ring", "device", 3, norm_every=1)

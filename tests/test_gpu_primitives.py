@@ -77,6 +77,53 @@ def test_put_signal_ring(P, nbytes):
             assert np.array_equal(o, (base + rnd).astype(np.uint8)), (rank, rnd)
 
 
+@pytest.mark.parametrize("P", [1, 2, 3])
+@pytest.mark.parametrize("nbytes,blocks", [(4096, 0), (1 << 20, 0), (1 << 20, 7), ((3 << 20) + 16, 0)])
+def test_p2p_bench_patterns_deliver_data(P, nbytes, blocks):
+    """uc_p2p_bench (configs[4] machinery): ping-pong and window move the sender's bytes into
+    the partner's landing zone; the halo pattern fills both neighbours' zones; repeated calls
+    keep the signal bases of every (pattern, peer) pair in step."""
+    import torch
+
+    def body(rank, P, ag):
+        U, env, comm, stream, coord = _setup(rank, P, ag, 1)
+        buf = U.SymMem(comm, 3 * nbytes)
+        sig = U.SymMem(comm, 64)
+        try:
+            with torch.cuda.stream(stream):
+                mine = dev_bytes(buf.ptr(), 3 * nbytes)
+                mine[:nbytes] = (torch.arange(nbytes, device="cuda", dtype=torch.int32) * (rank + 3) % 251).to(
+                    torch.uint8)
+            # never torch.cuda.synchronize() here: a device-wide sync in one virtual rank would
+            # wait for a peer's kernel that spins on this rank's not-yet-launched kernel
+            stream.synchronize()
+            comm.barrier()
+            got = {}
+            for rnd in range(2):
+                if P >= 2 and rank in (0, 1):
+                    coord.p2p_bench(U.UC_P2P_PINGPONG, buf, sig, nbytes, 3, 1, 1 - rank, rank, blocks)
+                    coord.p2p_bench(U.UC_P2P_WINDOW, buf, sig, nbytes, 2, 4, 1 - rank, rank, blocks)
+                coord.p2p_bench(U.UC_P2P_HALO, buf, sig, nbytes, 3, 1, 0, 0, blocks)
+                coord.sync()
+                comm.barrier()
+            got = mine.cpu().numpy()
+            comm.barrier()
+            return got
+        finally:
+            _teardown(env, comm, coord, buf, sig)
+
+    res = run_ranks(P, body)
+
+    def src(r):
+        return ((np.arange(nbytes, dtype=np.int64) * (r + 3)) % 251).astype(np.uint8)
+
+    for r in range(P):
+        top, bot = (r - 1) % P, (r + 1) % P
+        # halo: zone [bytes, 2 bytes) from top, [2 bytes, 3 bytes) from bottom
+        assert np.array_equal(res[r][nbytes:2 * nbytes], src(top)), r
+        assert np.array_equal(res[r][2 * nbytes:], src(bot)), r
+
+
 @pytest.mark.parametrize("dtype", ["f32", "f64", "u64"])
 @pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
 def test_allreduce_device_oneshot(P, dtype):
