@@ -60,6 +60,7 @@ def parse():
     ap.add_argument("--cpu-sample-iters", type=int, default=3)
     ap.add_argument("--variant", type=int, default=-1, help="0 register march, 1 TMA-staged (-1: library default)")
     ap.add_argument("--stages", type=int, default=0)
+    ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--block-x", type=int, default=0)
     ap.add_argument("--blocks-per-sm", type=int, default=0)
     return ap.parse_args()
@@ -189,8 +190,8 @@ def run_ours(a):
     stream = torch.cuda.Stream()
     coord = U.Coord(comm, mode, stream.cuda_stream)
     J = U.Jacobi(comm, nx, ny)
-    if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages:
-        J.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages)
+    if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages or a.tile_rows:
+        J.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages, a.tile_rows)
     n = J.n
     launch_info = J.launch_info()
     use_graph = not a.no_graph

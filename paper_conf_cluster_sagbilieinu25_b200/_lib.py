@@ -68,8 +68,8 @@ _SIGS = {
     "uc_jacobi_copy_out_async": (i32, [vp, vp, vp]),
     "uc_jacobi_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32), P(i64)]),
     "uc_jacobi_destroy": (i32, [vp]),
-    "uc_jacobi_set_launch": (i32, [vp, i32, i32, i32, i32]),
-    "uc_jacobi_launch_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32), P(i32), P(i32)]),
+    "uc_jacobi_set_launch": (i32, [vp, i32, i32, i32, i32, i32]),
+    "uc_jacobi_launch_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32), P(i32), P(i32), P(i32)]),
     "uc_last_error": (C.c_char_p, []),
     "uc_status_string": (C.c_char_p, [i32]),
     "uc_version": (i32, []),

@@ -260,6 +260,7 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
     }
     p.k_dev[0] = p.k_dev[0] + 1;
     *p.done = 0;
+    *p.work = 0;  // variant 2 tile counter
     __threadfence();
   }
 }
@@ -333,13 +334,141 @@ __device__ __forceinline__ void march_staged(const JacobiParams& p, const float*
   }
 }
 
+// ------------------------------------------------------------------------------ dynamic tiles
+// Variant 2: the staged ring of variant 1, but blocks pull (strip, row-tile) work items from a
+// device-wide counter instead of owning one fixed chunk, so faster SMs take more tiles and the
+// one-wave tail disappears.  Items are ordered tile-major (all strips of a row band are
+// consecutive), so concurrently processed items cover whole rows and the 2 halo rows a tile
+// shares with its vertical neighbours are usually still in L2.  The producer warp grabs the
+// items and tells the consumers what each ring stage holds through a per-stage header
+// (published by the mbarrier arrive, which has release semantics).
+struct StageHdr {
+  int y;   // slab row held by the stage; -1 = no more work
+  int y0;  // first computed row of the item
+  int s;   // strip
+  int pad;
+};
+
+template <bool NORM>
+__device__ __forceinline__ void march_dynamic(const JacobiParams& p, const float* src, float* dst, int r0, int r1,
+                                              double& acc, float* ring, uint64_t* full, uint64_t* empty,
+                                              StageHdr* hdr) {
+  const int nc = p.consumers, NS = p.stages;
+  const int ST = 4 * nc + 2 * kPad;
+  const int lane = threadIdx.x & 31;
+  const size_t pitch = (size_t)p.nx;
+  const int T = p.tile_rows;
+  const int tiles = r1 >= r0 ? (r1 - r0 + T) / T : 0;
+  const int total = tiles * p.strips;
+  if ((int)threadIdx.x >= nc) {
+    if (lane != 0) return;
+    // ---- producer
+#if UC_L2_EVICT_FIRST
+    const uint64_t pol = policy_evict_first();
+#else
+    const uint64_t pol = policy_evict_normal();
+#endif
+    // Item order "spread": the row range is cut into R = chunks regions; consecutive groups of
+    // S items take the next tile of every region in turn, so the tiles in flight are spread
+    // over the slab like the static chunks of variant 1 (which measured faster than marching
+    // one compact band), while the tail is still balanced dynamically.
+    const int R = max(1, min(p.chunks, tiles));
+    const int tpr = (tiles + R - 1) / R;  // tiles per region
+    const int slots = tpr * R * p.strips;
+    int i = 0;
+    for (;;) {
+      int item = (int)atomicAdd(p.work, 1u);
+      int tile = 0;
+      while (item < slots) {
+        const int j = item / p.strips;
+        tile = (j % R) * tpr + j / R;
+        if (tile < tiles) break;
+        item = (int)atomicAdd(p.work, 1u);  // an empty slot of the last region
+      }
+      const bool done = item >= slots || total == 0;
+      const int s = done ? 0 : item % p.strips;
+      const int y0 = done ? 0 : r0 + tile * T;
+      const int y1 = done ? -2 : min(y0 + T - 1, r1);
+      const int x0 = s * 4 * nc;
+      const int left = x0 >= kPad ? x0 - kPad : 0;
+      const int right = min(x0 + 4 * nc + kPad, p.nx);
+      const unsigned bytes = (unsigned)(right - left) * 4u;
+      const int off = left - (x0 - kPad);
+      for (int y = y0 - 1; y <= y1 + 1 || done; ++y, ++i) {
+        const int st = i % NS;
+        if (i >= NS) mbar_wait(empty + st, (unsigned)((i / NS) - 1) & 1u);
+        hdr[st] = StageHdr{done ? -1 : y, y0, s, 0};
+        if (done) {
+          mbar_arrive(full + st);  // header only, no bytes
+          return;
+        }
+        mbar_arrive_expect_tx(full + st, bytes);
+        bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)y * pitch + left, bytes, full + st, pol);
+      }
+    }
+  }
+  // ---- consumers
+  const int t = threadIdx.x;
+  float4 up = make_float4(0.f, 0.f, 0.f, 0.f), cur = up;
+  float ec = 0.f;
+  for (int i = 0;; ++i) {
+    const int st = i % NS;
+    mbar_wait(full + st, (unsigned)(i / NS) & 1u);
+    const StageHdr h = hdr[st];
+    if (h.y < 0) return;
+    const int x4 = h.s * nc + t;
+    const bool valid = x4 < p.nx4;
+    const float* row = ring + (size_t)st * ST + kPad + 4 * t;
+    const float4 v = *reinterpret_cast<const float4*>(row);
+    float e = 0.f;
+    if (lane == 0) e = row[-1];
+    else if (lane == 31) e = row[4];
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty + st);
+    if (h.y == h.y0 - 1) {
+      up = v;
+    } else if (h.y == h.y0) {
+      cur = v;
+      ec = e;
+    } else {
+      const int y = h.y - 1;
+      const float4 o = row_update(up, cur, v, ec, lane, x4, p.nx4);
+      if (valid) st4(dst + (size_t)y * pitch + 4 * (size_t)x4, o);
+      if (NORM && valid) acc_sq(acc, o, cur);
+      up = cur;
+      cur = v;
+      ec = e;
+    }
+  }
+}
+
 // ------------------------------------------------------------------------------ the kernel
 template <int VARIANT, bool NORM>
 __device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t k, float* ring, uint64_t* full,
-                                                 uint64_t* empty) {
+                                                 uint64_t* empty, StageHdr* hdr) {
   const int par = (int)(k & 1);
   const float* src = p.slab[par];
   float* dst = p.slab[par ^ 1];
+  if (VARIANT == 2) {
+    double acc = 0.0;
+    const int lane = threadIdx.x & 31;
+    const int nc = p.consumers;
+    int r0 = 1, r1 = p.n;
+    if (p.device_mode) {
+      // boundary work items first: blocks [0, S) row 1 of strip b, [S, 2S) row n (n >= 2)
+      const int nb = p.n >= 2 ? 2 * p.strips : p.strips;
+      for (int j = blockIdx.x; j < nb; j += gridDim.x) {
+        const int s = j % p.strips;
+        const int x4 = (int)threadIdx.x < nc ? s * nc + (int)threadIdx.x : 0x3fffffff;
+        if (j < p.strips) boundary_row<NORM>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
+        else boundary_row<NORM>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+      }
+      r0 = 2;
+      r1 = p.n - 1;
+    }
+    march_dynamic<NORM>(p, src, dst, r0, r1, acc, ring, full, empty, hdr);
+    return acc;
+  }
   const int s = blockIdx.x % p.strips;
   const int q = blockIdx.x / p.strips;
   const int lane = threadIdx.x & 31;
@@ -371,11 +500,13 @@ __global__ void __launch_bounds__(kMaxBlock + 32, UC_MINBLOCKS) jacobi_iter_kern
   extern __shared__ __align__(128) unsigned char dyn[];
   float* ring = nullptr;
   uint64_t *full = nullptr, *empty = nullptr;
-  if (VARIANT == 1) {
+  StageHdr* hdr = nullptr;
+  if (VARIANT >= 1) {
     const int NS = p.stages;
     full = reinterpret_cast<uint64_t*>(dyn);
     empty = full + NS;
-    ring = reinterpret_cast<float*>(dyn + ((16 * NS + 127) / 128) * 128);  // after 2*NS mbarriers
+    hdr = reinterpret_cast<StageHdr*>(empty + NS);
+    ring = reinterpret_cast<float*>(dyn + ((32 * NS + 127) / 128) * 128);  // after mbarriers + headers
     if (threadIdx.x == 0) {
       for (int i = 0; i < NS; ++i) {
         mbar_init(full + i, 1);                   // the producer's arrive.expect_tx
@@ -388,11 +519,11 @@ __global__ void __launch_bounds__(kMaxBlock + 32, UC_MINBLOCKS) jacobi_iter_kern
   const uint64_t k = p.k_dev[0];
   const bool do_norm = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
   if (do_norm) {
-    const double acc = iteration_body<VARIANT, true>(p, k, ring, full, empty);
+    const double acc = iteration_body<VARIANT, true>(p, k, ring, full, empty, hdr);
     const double t = block_sum(acc, smem);
     if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
   } else {
-    iteration_body<VARIANT, false>(p, k, ring, full, empty);
+    iteration_body<VARIANT, false>(p, k, ring, full, empty, hdr);
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -686,14 +817,17 @@ __global__ void allreduce_oneshot_kernel(const void* send, void* recv, size_t co
 
 // ------------------------------------------------------------------------------ launchers
 size_t staged_smem_bytes(int consumers, int stages) {
-  return (size_t)((16 * stages + 127) / 128) * 128 + (size_t)stages * (4 * consumers + 2 * kPad) * sizeof(float);
+  // [full mbarriers][empty mbarriers][stage headers] padded to 128 B, then the row ring
+  return (size_t)((32 * stages + 127) / 128) * 128 + (size_t)stages * (4 * consumers + 2 * kPad) * sizeof(float);
 }
 
-int launch_jacobi_iteration(const JacobiParams& p, int block, cudaStream_t s) {
-  if (p.variant == 1)
-    jacobi_iter_kernel<1><<<p.strips * p.chunks, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p);
+int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s) {
+  if (p.variant == 2)
+    jacobi_iter_kernel<2><<<grid, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p);
+  else if (p.variant == 1)
+    jacobi_iter_kernel<1><<<grid, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p);
   else
-    jacobi_iter_kernel<0><<<p.strips * p.chunks, block, 0, s>>>(p);
+    jacobi_iter_kernel<0><<<grid, block, 0, s>>>(p);
   UC_CUDA(cudaGetLastError());
   return UC_OK;
 }
@@ -755,7 +889,9 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
 // mode) must never depend on such a load happening concurrently.
 int preload_kernels() {
   UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
   const void* fns[] = {(const void*)jacobi_iter_kernel<0>, (const void*)jacobi_iter_kernel<1>,
+                       (const void*)jacobi_iter_kernel<2>,
                        (const void*)norm_finish_kernel,
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
@@ -769,7 +905,9 @@ int preload_kernels() {
 }
 
 int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm) {
-  if (variant == 1)
+  if (variant == 2)
+    UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<2>, block, smem));
+  else if (variant == 1)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<1>, block, smem));
   else
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<0>, block, 0));

@@ -53,6 +53,8 @@ struct JacobiParams {
   uint64_t* norm_flag[UC_MAX_RANKS];   // rank q's norm flags: [2][P] u64 (stride kFlagStride)
   unsigned long long* k_dev;           // local iteration counter
   unsigned int* done;                  // local block ticket
+  unsigned int* work;                  // local dynamic tile counter (variant 2)
+  int tile_rows;                       // variant 2: rows per work item
   double* partials;                    // local [grid] per-block partial sums
   double* rank_sum;                    // local: this rank's sum of squares (host-mode allreduce in place)
   double* norm_hist;                   // local: norms by round m (ring of norm_cap)
@@ -77,9 +79,10 @@ constexpr int kFlagStride = 16;  // u64 per flag = 128 bytes, one flag per L2 li
 // with a 3-row ring reaches 6.36 TB/s vs 6.07 for the register march; deeper rings lose.
 constexpr int kDefaultVariant = 1;
 constexpr int kDefaultStages = 3;
+constexpr int kDefaultTileRows = 64;
 
 // Launch wrappers implemented in kernels.cu
-int launch_jacobi_iteration(const JacobiParams& p, int block, cudaStream_t s);
+int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
 int launch_init_field(float* slab0, float* slab1, int nx, int n, int ny, int row0, int ring,
@@ -192,7 +195,7 @@ struct uc_jacobi {
   double* norm_hist = nullptr;
   int norm_cap = 4096;
   cudaStream_t aux = nullptr;    // private non-blocking stream (init, synchronous copies)
-  int variant = uc::kDefaultVariant, consumers = 0, stages = 0;
+  int variant = uc::kDefaultVariant, consumers = 0, stages = 0, tile_rows = 0;
   int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
   int partials_cap = 0;
   std::vector<JacobiGraph> graphs;

@@ -249,16 +249,18 @@ class Jacobi:
     def copy_out_async(self, coord: Coord, host_ptr: int):
         check(lib.uc_jacobi_copy_out_async(coord.h, self.h, C.c_void_p(host_ptr)), "uc_jacobi_copy_out_async")
 
-    def set_launch(self, variant: int = -1, block_x: int = 0, blocks_per_sm: int = 0, stages: int = 0):
+    def set_launch(self, variant: int = -1, block_x: int = 0, blocks_per_sm: int = 0, stages: int = 0,
+                   tile_rows: int = 0):
         """COLLECTIVE (see uc_jacobi_set_launch)."""
-        check(lib.uc_jacobi_set_launch(self.h, variant, block_x, blocks_per_sm, stages), "uc_jacobi_set_launch")
+        check(lib.uc_jacobi_set_launch(self.h, variant, block_x, blocks_per_sm, stages, tile_rows),
+              "uc_jacobi_set_launch")
 
     def launch_info(self) -> dict:
-        v, g, b, s, c, st = (C.c_int() for _ in range(6))
+        v, g, b, s, c, st, tr = (C.c_int() for _ in range(7))
         check(lib.uc_jacobi_launch_info(self.h, C.byref(v), C.byref(g), C.byref(b), C.byref(s), C.byref(c),
-                                        C.byref(st)), "uc_jacobi_launch_info")
+                                        C.byref(st), C.byref(tr)), "uc_jacobi_launch_info")
         return {"variant": v.value, "grid": g.value, "block": b.value, "strips": s.value, "chunks": c.value,
-                "stages": st.value}
+                "stages": st.value, "tile_rows": tr.value}
 
     def destroy(self):
         if self.h:

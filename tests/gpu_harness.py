@@ -16,7 +16,7 @@ def neighbours(U, topology):
 
 def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0, seed=gen.DEFAULT_SEED,
               zero_init=False, init=None, use_graph=True, stepwise=False, block_x=0, blocks_per_sm=0,
-              variant=-1, stages=0,
+              variant=-1, stages=0, tile_rows=0,
               chunks_of_run=None):
     """Returns dict(init=[slab0 per rank], final=[slab per rank], norms=np.array (rank 0),
     norms_all=[per rank], launch=launch_info of rank 0)."""
@@ -33,8 +33,8 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
         coord.set_timeout(5.0)
         J = U.Jacobi(comm, nx, ny, seed, zero_init)
         try:
-            if block_x or blocks_per_sm or variant >= 0 or stages:
-                J.set_launch(variant, block_x, blocks_per_sm, stages)
+            if block_x or blocks_per_sm or variant >= 0 or stages or tile_rows:
+                J.set_launch(variant, block_x, blocks_per_sm, stages, tile_rows)
             slab0 = J.copy_out()
             if init is not None:
                 J.copy_in(gen.rank_slab(init, rank, P))

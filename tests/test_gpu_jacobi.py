@@ -99,31 +99,36 @@ def test_graph_and_stepwise_agree():
     assert np.array_equal(a["norms"], c["norms"][[0, 7, 14, 21, 28]])
 
 
-@pytest.mark.parametrize("variant", [0, 1])
-@pytest.mark.parametrize("block_x,bps,stages", [(32, 1, 3), (64, 2, 4), (128, 0, 0), (256, 1, 16)])
-def test_launch_geometries(variant, block_x, bps, stages):
-    """Both kernel variants, different block widths / chunk counts / ring depths change the
-    blocking, not the results."""
+@pytest.mark.parametrize("variant", [0, 1, 2])
+@pytest.mark.parametrize("block_x,bps,stages,tile", [(32, 1, 3, 5), (64, 2, 4, 1), (128, 0, 0, 0), (256, 1, 16, 33)])
+def test_launch_geometries(variant, block_x, bps, stages, tile):
+    """All kernel variants, different block widths / chunk counts / ring depths / tile heights
+    change the blocking, not the results."""
     res = _check(1024, 96, 1, "ring", "device", 9, norm_every=3, block_x=block_x, blocks_per_sm=bps,
-                 variant=variant, stages=stages)
-    assert res["launch"]["block"] == block_x + (32 if variant == 1 else 0)
+                 variant=variant, stages=stages, tile_rows=tile)
+    assert res["launch"]["block"] == block_x + (32 if variant >= 1 else 0)
     assert res["launch"]["variant"] == variant
 
 
-STAGED = dict(variant=1)
-
-
+@pytest.mark.parametrize("variant", [1, 2])
 @pytest.mark.parametrize("topology", ["ring", "dirichlet"])
 @pytest.mark.parametrize("mode", ["device", "host"])
-def test_staged_variant_c1(topology, mode):
-    _check(256, 256, 1, topology, mode, 100, norm_every=10, **STAGED)
+def test_staged_variants_c1(variant, topology, mode):
+    _check(256, 256, 1, topology, mode, 100, norm_every=10, variant=variant)
 
 
+@pytest.mark.parametrize("variant,tile", [(1, 0), (2, 0), (2, 3)])
 @pytest.mark.parametrize("nx,ny,P", [(1028, 64, 1), (4, 2, 1), (2052, 33, 1), (520, 96, 4), (64, 3, 3),
                                      (36, 16, 8)])
-def test_staged_variant_shapes(nx, ny, P):
+def test_staged_variants_shapes(nx, ny, P, variant, tile):
     for topology in ("ring", "dirichlet"):
-        _check(nx, ny, P, topology, "device", 13, norm_every=4, **STAGED)
+        _check(nx, ny, P, topology, "device", 13, norm_every=4, variant=variant, tile_rows=tile)
+
+
+@pytest.mark.parametrize("variant", [0, 1, 2])
+def test_full_size_each_variant(variant):
+    """16384^2, device mode, 3 iterations, whole grid bit-exact for every kernel variant."""
+    _check(16384, 16384, 1, "ring", "device", 3, norm_every=1, variant=variant)
 
 
 def test_switch_variant_mid_run():
