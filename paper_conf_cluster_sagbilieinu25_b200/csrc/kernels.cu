@@ -174,13 +174,16 @@ __device__ __forceinline__ void march(const float* __restrict__ src, float* __re
 // Device mode: the fused compute + put + signal of one boundary row for strip s (Listing 3,
 // P:55-68; §8 a3).  top_side: row y == 1 goes to the top neighbour's halo row n+1;
 // bot_side: row y == n goes to the bottom neighbour's halo row 0.  Both when n == 1.
+// PartialDevice mode (device_mode == 2, Listing 6): the same puts without waits or
+// signals; the host-side Acknowledge after the kernel synchronises the neighbours.
 template <bool NORM>
 __device__ __forceinline__ void boundary_row(const JacobiParams& p, const float* src, float* dst, int y, int x4,
                                              int lane, int s, uint64_t k, bool top_side, bool bot_side,
                                              double& acc) {
   const bool put_top = top_side && p.has_top;
   const bool put_bot = bot_side && p.has_bot;
-  if (threadIdx.x == 0) {
+  const bool fused = p.device_mode == 1;
+  if (threadIdx.x == 0 && fused) {
     // halo rows of A_k (slab k&1) must hold the neighbours' A_k rows: wait for flag >= k
     if (put_top) wait_ge(p.my_flags + (size_t)s * kFlagStride, k, p.timeout_ns, p.err);
     if (put_bot) wait_ge(p.my_flags + (size_t)(p.flag_half + s) * kFlagStride, k, p.timeout_ns, p.err);
@@ -201,7 +204,7 @@ __device__ __forceinline__ void boundary_row(const JacobiParams& p, const float*
     if (put_bot) reinterpret_cast<float4*>(p.bot_slab[np])[x4] = o;
   }
   if (NORM && valid) acc_sq(acc, o, cur);
-  if (put_top || put_bot) {
+  if (fused && (put_top || put_bot)) {
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence_system();
@@ -238,7 +241,7 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
   }
   if (threadIdx.x == 0) {
     if (do_norm) {
-      if (p.device_mode) {
+      if (p.device_mode == 1) {
         // one-shot P2P allreduce of the rank partial (§8 a5): write slot[rank] on every rank,
         // release a flag, wait for all P flags, sum slots 0..P-1 in rank order (reading G12).
         const uint64_t m = p.k_dev[1];
@@ -255,7 +258,7 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
         p.norm_hist[m % (uint64_t)p.norm_cap] = sqrt(g);
         p.k_dev[1] = m + 1;
       } else {
-        *p.rank_sum = tot;  // host mode: ncclAllReduce + norm_finish_kernel complete it
+        *p.rank_sum = tot;  // host/partial mode: ncclAllReduce + norm_finish_kernel complete it
       }
     }
     p.k_dev[0] = p.k_dev[0] + 1;
@@ -741,6 +744,37 @@ int launch_p2p_bench(const P2PLaunch& L, cudaStream_t s) {
   return UC_OK;
 }
 
+// PartialDevice Acknowledge (P:198-203 with P:277-279): after the stencil kernel of iteration
+// k posted its boundary rows to the neighbours without signals, this stream-ordered kernel
+// tells both neighbours "my iteration k is complete" (flags = k+1 for every strip, so device
+// mode can follow) and waits until both neighbours say the same.  Afterwards the halo rows of
+// A_{k+1} are in place and the neighbours have finished reading the slab we will write next.
+// The completed iteration count is read from the device counter (already bumped by the
+// stencil kernel), so graph replays stay correct.
+__global__ void partial_ack_kernel(uint64_t* my_flags, uint64_t* top_flags, uint64_t* bot_flags, int strips,
+                                   int flag_half, const unsigned long long* k_dev, unsigned long long timeout_ns,
+                                   unsigned int* err) {
+  const uint64_t v = k_dev[0];  // = k + 1
+  __threadfence_system();
+  __syncthreads();
+  for (int s = threadIdx.x; s < strips; s += blockDim.x) {
+    if (top_flags) st_release_sys(top_flags + (size_t)(flag_half + s) * kFlagStride, v);
+    if (bot_flags) st_release_sys(bot_flags + (size_t)s * kFlagStride, v);
+  }
+  for (int s = threadIdx.x; s < strips; s += blockDim.x) {
+    if (top_flags) wait_ge(my_flags + (size_t)s * kFlagStride, v, timeout_ns, err);
+    if (bot_flags) wait_ge(my_flags + (size_t)(flag_half + s) * kFlagStride, v, timeout_ns, err);
+  }
+}
+
+int launch_partial_ack(uint64_t* my_flags, uint64_t* top_flags, uint64_t* bot_flags, int strips, int flag_half,
+                       const unsigned long long* k_dev, unsigned long long timeout_ns, unsigned int* err,
+                       cudaStream_t s) {
+  partial_ack_kernel<<<1, 128, 0, s>>>(my_flags, top_flags, bot_flags, strips, flag_half, k_dev, timeout_ns, err);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
 // Device mode: the halo rows of the current iterate A_k are written by the neighbours during
 // THEIR iteration k-1, possibly after this rank finished its own; before the slab is read back
 // the stream waits for every per-strip flag >= k.
@@ -896,6 +930,7 @@ int preload_kernels() {
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
                        (const void*)wait_halo_kernel,   (const void*)p2p_bench_kernel,
+                       (const void*)partial_ack_kernel,
                        (const void*)uc_fill_f32};
   for (const void* f : fns) {
     cudaFuncAttributes a;

@@ -330,12 +330,29 @@ int uc_mem_free_symmetric(uc_mem* m) {
   return UC_OK;
 }
 
+}  // extern "C"
+
+// NCCL communicator of a coordinator, created on first need (COLLECTIVE: every rank reaches
+// it through the same collective call; the unique id travels over the bootstrap allgather).
+int uc::ensure_nccl(uc_coord* k) {
+  if (k->nccl) return UC_OK;
+  uc_comm* c = k->comm;
+  ncclUniqueId id{};
+  if (c->rank == 0) UC_NCCL(ncclGetUniqueId(&id));
+  std::vector<ncclUniqueId> ids(c->size);
+  UC_TRY(c->env->allgather(&id, ids.data(), sizeof id));
+  UC_NCCL(ncclCommInitRank(&k->nccl, c->size, ids[0], c->rank));
+  return UC_OK;
+}
+
+extern "C" {
+
 // ============================================================================ Coordinator
 int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
   if (!c || !out) return fail(UC_ERR_ARG, "NULL argument");
   *out = nullptr;
-  if (mode == UC_MODE_PARTIAL) return fail(UC_ERR_UNSUPPORTED, "PartialDevice launch mode is not implemented yet");
-  if (mode != UC_MODE_HOST && mode != UC_MODE_DEVICE) return fail(UC_ERR_ARG, "unknown mode %d", (int)mode);
+  if (mode != UC_MODE_HOST && mode != UC_MODE_DEVICE && mode != UC_MODE_PARTIAL)
+    return fail(UC_ERR_ARG, "unknown mode %d", (int)mode);
   if (c->env->device < 0) return fail(UC_ERR_STATE, "bootstrap-only environment has no device");
   UC_CUDA(cudaSetDevice(c->env->device));
   uc_coord* k = new uc_coord;
@@ -356,18 +373,13 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
   k->p2p_bar = k->put_counter + 1;
   if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
   if (e != cudaSuccess) return cleanup(fail(UC_ERR_CUDA, "coordinator state: %s", cudaGetErrorString(e)));
+  // host mode: NCCL for everything; partial mode: NCCL for collectives, created at the
+  // first collective, + peer memory for the in-kernel posts; device mode: peer memory only
   if (mode == UC_MODE_HOST) {
-    ncclUniqueId id{};
-    if (c->rank == 0) {
-      ncclResult_t r = ncclGetUniqueId(&id);
-      if (r != ncclSuccess) return cleanup(fail(UC_ERR_NCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r)));
-    }
-    std::vector<ncclUniqueId> ids(c->size);
-    int rc = c->env->allgather(&id, ids.data(), sizeof id);
+    int rc = ensure_nccl(k);
     if (rc != UC_OK) return cleanup(rc);
-    ncclResult_t r = ncclCommInitRank(&k->nccl, c->size, ids[0], c->rank);
-    if (r != ncclSuccess) return cleanup(fail(UC_ERR_NCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
-  } else {
+  }
+  if (mode != UC_MODE_HOST) {
     const size_t P = (size_t)c->size;
     const size_t bytes = 2 * P * k->ar_slot_bytes + 2 * P * kFlagStride * sizeof(uint64_t);
     int rc = uc_mem_alloc_symmetric(c, bytes, &k->ar_scratch);
@@ -519,7 +531,7 @@ int uc_signal_wait(uc_coord* k, uc_mem* dst, size_t dst_off, size_t bytes, uc_me
 int uc_p2p_bench(uc_coord* k, int pattern, uc_mem* buf, uc_mem* sig, size_t bytes, int iters, int window, int peer,
                  int role, int blocks) {
   if (!k || !buf || !sig) return fail(UC_ERR_ARG, "NULL argument");
-  if (k->mode != UC_MODE_DEVICE) return fail(UC_ERR_UNSUPPORTED, "uc_p2p_bench runs device-initiated patterns only");
+  if (k->mode == UC_MODE_HOST) return fail(UC_ERR_UNSUPPORTED, "uc_p2p_bench runs device-initiated patterns only");
   if (pattern < UC_P2P_PINGPONG || pattern > UC_P2P_HALO) return fail(UC_ERR_ARG, "unknown pattern %d", pattern);
   if (bytes == 0 || bytes % 16) return fail(UC_ERR_ARG, "bytes must be a positive multiple of 16");
   if (iters < 1 || (pattern == UC_P2P_WINDOW && window < 1)) return fail(UC_ERR_ARG, "iters/window must be >= 1");
@@ -575,7 +587,8 @@ int uc_allreduce_sum(uc_coord* k, const void* send, void* recv, size_t count, uc
   uc_comm* c = k->comm;
   UC_CUDA(cudaSetDevice(c->env->device));
   if (count == 0) return UC_OK;
-  if (k->mode == UC_MODE_HOST) {
+  if (k->mode != UC_MODE_DEVICE) {  // host mode, and partial mode ("collectives as PureHost")
+    UC_TRY(ensure_nccl(k));
     ncclDataType_t t = dt == UC_F32 ? ncclFloat32 : dt == UC_F64 ? ncclFloat64 : ncclUint64;
     UC_NCCL(ncclAllReduce(send, recv, count, t, ncclSum, k->nccl, k->stream));
     return UC_OK;

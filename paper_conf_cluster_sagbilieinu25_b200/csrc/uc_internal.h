@@ -109,10 +109,14 @@ struct P2PLaunch {
   unsigned int* err;
 };
 int launch_p2p_bench(const P2PLaunch& L, cudaStream_t s);
+int launch_partial_ack(uint64_t* my_flags, uint64_t* top_flags, uint64_t* bot_flags, int strips, int flag_half,
+                       const unsigned long long* k_dev, unsigned long long timeout_ns, unsigned int* err,
+                       cudaStream_t s);
 int launch_wait_halo(const uint64_t* my_flags, int strips, int flag_half, int has_top, int has_bot, uint64_t k,
                      unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 size_t staged_smem_bytes(int consumers, int stages);
 int preload_kernels();
+int ensure_nccl(uc_coord* k);
 const void* builtin_kernel(const char* name);
 
 }  // namespace uc
@@ -196,6 +200,7 @@ struct uc_jacobi {
   int norm_cap = 4096;
   cudaStream_t aux = nullptr;    // private non-blocking stream (init, synchronous copies)
   int variant = uc::kDefaultVariant, consumers = 0, stages = 0, tile_rows = 0;
+  int last_mode = -1;            // mode of the coordinator that ran the previous iterations
   int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
   int partials_cap = 0;
   std::vector<JacobiGraph> graphs;

@@ -7,7 +7,7 @@ import numpy as np
 from inputs import gen
 from vranks import run_ranks
 
-MODES = {"device": 1, "host": 0}
+MODES = {"device": 1, "host": 0, "partial": 2}
 
 
 def neighbours(U, topology):

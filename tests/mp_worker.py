@@ -38,7 +38,8 @@ def main():
     neigh = U.ring_neighbours if a.topology == "ring" else U.chain_neighbours
     comm = U.Comm(env, *neigh(rank, world))
     stream = torch.cuda.Stream()
-    coord = U.Coord(comm, U.UC_MODE_DEVICE if a.mode == "device" else U.UC_MODE_HOST, stream.cuda_stream)
+    mode = {"device": U.UC_MODE_DEVICE, "host": U.UC_MODE_HOST, "partial": U.UC_MODE_PARTIAL}[a.mode]
+    coord = U.Coord(comm, mode, stream.cuda_stream)
     coord.set_timeout(20.0)
     J = U.Jacobi(comm, a.nx, a.ny)
     norms = J.run(coord, a.iters, a.norm_every, use_graph=True)

@@ -87,6 +87,44 @@ def test_host_mode_single_rank_nccl_self_exchange():
     _check(1028, 50, 1, "ring", "host", 13, norm_every=3)
 
 
+@pytest.mark.parametrize("variant", [0, 1, 2])
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+def test_partial_device_mode(variant, topology):
+    """PartialDevice (Listing 6): in-kernel posts without signals + stream-ordered
+    Acknowledge.  P = 1 with norms (NCCL allreduce, single rank); P = 2..4 virtual ranks
+    without norms (two NCCL ranks cannot share one GPU)."""
+    _check(1028, 48, 1, topology, "partial", 17, norm_every=4, variant=variant)
+    for P in (2, 3, 4):
+        _check(1028, 48, P, topology, "partial", 17, norm_every=0, variant=variant)
+
+
+def test_modes_interchangeable_on_one_solver():
+    """Device, partial and (P = 1) host iterations can follow each other on one solver."""
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+    nx, ny = 520, 40
+    env = U.Env(0, 1, 0)
+    comm = U.Comm(env, 0, 0)
+    st = torch.cuda.Stream()
+    coords = {m: U.Coord(comm, MODES_[m], st.cuda_stream) for m in ("device", "partial", "host")}
+    J = U.Jacobi(comm, nx, ny)
+    for m in ("device", "partial", "host", "device", "partial"):
+        J.run(coords[m], 5, 0)
+        coords[m].sync()
+    out = J.copy_out(coords["device"])
+    J.destroy()
+    for c in coords.values():
+        c.destroy()
+    comm.destroy()
+    env.finalize()
+    _, want, _ = _oracle(nx, ny, "ring", 25, 0)
+    assert np.array_equal(bits(out), bits(gen.rank_slab(want, 0, 1)))
+
+
+MODES_ = {"device": 1, "host": 0, "partial": 2}
+
+
 def test_graph_and_stepwise_agree():
     a = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=True)
     b = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=False)

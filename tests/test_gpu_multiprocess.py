@@ -27,13 +27,15 @@ def _port():
     return p
 
 
-@pytest.mark.parametrize("P,topology", [(2, "ring"), (3, "dirichlet"), (4, "ring")])
-def test_multiprocess_ipc_device_mode(tmp_path, P, topology):
-    nx, ny, iters, ne = 520, 16 * P, 20, 5
+@pytest.mark.parametrize("P,topology,mode", [(2, "ring", "device"), (3, "dirichlet", "device"), (4, "ring", "device"),
+                                             (3, "ring", "partial")])
+def test_multiprocess_ipc_device_mode(tmp_path, P, topology, mode):
+    nx, ny, iters = 520, 16 * P, 20
+    ne = 5 if mode == "device" else 0  # partial-mode norms need NCCL: one GPU per rank
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={P}",
            "--master-addr", "127.0.0.1", "--master-port", str(_port()),
            os.path.join(ROOT, "tests", "mp_worker.py"), "--nx", str(nx), "--ny", str(ny), "--iters", str(iters),
-           "--norm-every", str(ne), "--topology", topology, "--same-device", "--out", str(tmp_path)]
+           "--norm-every", str(ne), "--topology", topology, "--mode", mode, "--same-device", "--out", str(tmp_path)]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=240, cwd=ROOT)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     res = [np.load(os.path.join(tmp_path, f"rank{q}.npz")) for q in range(P)]

@@ -212,11 +212,20 @@ def test_signal_wait_timeout_is_reported():
     assert run_ranks(1, body) == [True]
 
 
-def test_partial_mode_unsupported():
-    import paper_conf_cluster_sagbilieinu25_b200 as U
-    env = U.Env(0, 1, 0)
-    comm = U.Comm(env, 0, 0)
-    with pytest.raises(U.UCError, match="UNSUPPORTED"):
-        U.Coord(comm, U.UC_MODE_PARTIAL, 0)
-    comm.destroy()
-    env.finalize()
+def test_partial_mode_collectives_use_host_api():
+    """PartialDevice: collectives behave as PureHost -> NCCL, created on first use."""
+    import torch
+
+    def body(rank, P, ag):
+        U, env, comm, stream, coord = _setup(rank, P, ag, 2)
+        try:
+            with torch.cuda.stream(stream):
+                x = torch.arange(10, device="cuda", dtype=torch.float64)
+            coord.allreduce_sum(x.data_ptr(), x.data_ptr(), 10, 1)
+            coord.sync()
+            return x.cpu().numpy()
+        finally:
+            _teardown(env, comm, coord)
+
+    (x,) = run_ranks(1, body)
+    assert np.array_equal(x, np.arange(10, dtype=np.float64))
