@@ -231,6 +231,29 @@ __device__ __forceinline__ double block_sum(double v, double* smem) {
   return t;  // valid in thread 0
 }
 
+// Thread 0 of the block that summed the rank's partials: publish the norm round.
+__device__ void norm_publish(const JacobiParams& p, double tot) {
+  if (p.device_mode == 1) {
+    // one-shot P2P allreduce of the rank partial (§8 a5): write slot[rank] on every rank,
+    // release a flag, wait for all P flags, sum slots 0..P-1 in rank order (reading G12).
+    const uint64_t m = p.k_dev[1];
+    const int par = (int)(m & 1);
+    for (int q = 0; q < p.size; ++q) st_relaxed_sys_f64(p.norm_slot[q] + par * p.size + p.rank, tot);
+    __threadfence_system();
+    for (int q = 0; q < p.size; ++q)
+      st_release_sys(p.norm_flag[q] + (size_t)(par * p.size + p.rank) * kFlagStride, m + 1);
+    double g = 0.0;
+    for (int q = 0; q < p.size; ++q) {
+      wait_ge(p.norm_flag[p.rank] + (size_t)(par * p.size + q) * kFlagStride, m + 1, p.timeout_ns, p.err);
+      g += ld_relaxed_sys_f64(p.norm_slot[p.rank] + par * p.size + q);
+    }
+    p.norm_hist[m % (uint64_t)p.norm_cap] = sqrt(g);
+    p.k_dev[1] = m + 1;
+  } else {
+    *p.rank_sum = tot;  // host/partial mode: ncclAllReduce + norm_finish_kernel complete it
+  }
+}
+
 // Last block: deterministic sum of the block partials, cross-rank norm (device mode), counter bumps.
 __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* smem) {
   double tot = 0.0;
@@ -240,27 +263,7 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
     tot = block_sum(v, smem);
   }
   if (threadIdx.x == 0) {
-    if (do_norm) {
-      if (p.device_mode == 1) {
-        // one-shot P2P allreduce of the rank partial (§8 a5): write slot[rank] on every rank,
-        // release a flag, wait for all P flags, sum slots 0..P-1 in rank order (reading G12).
-        const uint64_t m = p.k_dev[1];
-        const int par = (int)(m & 1);
-        for (int q = 0; q < p.size; ++q) st_relaxed_sys_f64(p.norm_slot[q] + par * p.size + p.rank, tot);
-        __threadfence_system();
-        for (int q = 0; q < p.size; ++q)
-          st_release_sys(p.norm_flag[q] + (size_t)(par * p.size + p.rank) * kFlagStride, m + 1);
-        double g = 0.0;
-        for (int q = 0; q < p.size; ++q) {
-          wait_ge(p.norm_flag[p.rank] + (size_t)(par * p.size + q) * kFlagStride, m + 1, p.timeout_ns, p.err);
-          g += ld_relaxed_sys_f64(p.norm_slot[p.rank] + par * p.size + q);
-        }
-        p.norm_hist[m % (uint64_t)p.norm_cap] = sqrt(g);
-        p.k_dev[1] = m + 1;
-      } else {
-        *p.rank_sum = tot;  // host/partial mode: ncclAllReduce + norm_finish_kernel complete it
-      }
-    }
+    if (do_norm) norm_publish(p, tot);
     p.k_dev[0] = p.k_dev[0] + 1;
     *p.done = 0;
     *p.work = 0;  // variant 2 tile counter
@@ -275,10 +278,12 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
 // landed) and "empty" (all consumer warps copied the row out) per stage.  Up to NS-1 rows per
 // block are in flight without costing registers, which is what keeps HBM busy.
 // Ring layout: stage i = floats [i*ST, (i+1)*ST), ST = 4*nc + 8; column x0 - 4 sits at 0.
+// i0 = ring uses so far in this launch (the mbarrier phases continue from there); returns the
+// new count.
 template <bool NORM>
-__device__ __forceinline__ void march_staged(const JacobiParams& p, const float* src, float* dst, int s,
-                                             int x4, bool valid, int y0, int y1, double& acc, float* ring,
-                                             uint64_t* full, uint64_t* empty) {
+__device__ __forceinline__ int march_staged(const JacobiParams& p, const float* src, float* dst, int s, int x4,
+                                            bool valid, int y0, int y1, double& acc, float* ring, uint64_t* full,
+                                            uint64_t* empty, int i0 = 0, bool proxy_fence = false) {
   const int nc = p.consumers, NS = p.stages;
   const int ST = 4 * nc + 2 * kPad;
   const int lane = threadIdx.x & 31;
@@ -297,22 +302,27 @@ __device__ __forceinline__ void march_staged(const JacobiParams& p, const float*
 #else
       const uint64_t pol = policy_evict_normal();
 #endif
+      // rows written by generic-proxy stores earlier in this launch (persistent kernel) must be
+      // ordered before the async-proxy (TMA) reads
+      if (proxy_fence) fence_proxy_async_global();
       for (int i = 0; i < rows; ++i) {
-        const int st = i % NS;
-        if (i >= NS) mbar_wait(empty + st, (unsigned)((i / NS) - 1) & 1u);
+        const int g = i0 + i;  // ring use counter (continues across the iterations of a launch)
+        const int st = g % NS;
+        if (g >= NS) mbar_wait(empty + st, (unsigned)((g / NS) - 1) & 1u);
         mbar_arrive_expect_tx(full + st, bytes);
         bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(y0 - 1 + i) * pitch + left, bytes, full + st, pol);
       }
     }
-    return;
+    return i0 + rows;
   }
   // ---- consumer warps: copy the new row out of the ring, release the stage, compute
   const int t = threadIdx.x;
   float4 up = make_float4(0.f, 0.f, 0.f, 0.f), cur = up;
   float ec = 0.f;
   for (int i = 0; i < rows; ++i) {
-    const int st = i % NS;
-    mbar_wait(full + st, (unsigned)(i / NS) & 1u);
+    const int g = i0 + i;
+    const int st = g % NS;
+    mbar_wait(full + st, (unsigned)(g / NS) & 1u);
     const float* row = ring + (size_t)st * ST + kPad + 4 * t;
     const float4 v = *reinterpret_cast<const float4*>(row);
     float e = 0.f;
@@ -335,6 +345,7 @@ __device__ __forceinline__ void march_staged(const JacobiParams& p, const float*
       ec = e;
     }
   }
+  return i0 + rows;
 }
 
 // ------------------------------------------------------------------------------ dynamic tiles
@@ -539,6 +550,133 @@ __global__ void __launch_bounds__(kMaxBlock + 32, UC_MINBLOCKS) jacobi_iter_kern
     __threadfence();
     finish_iteration(p, do_norm, smem);
   }
+}
+
+// ------------------------------------------------------------------------------ persistent
+// Variant 3 ("CPU-free" Jacobi; the paper launches its device-API kernel with
+// nvshmemx_collective_launch): ONE launch runs `iters` iterations.  Every block keeps
+// its (strip, chunk) of variant 1 and its TMA ring across iterations; instead of a kernel
+// boundary (a device-wide barrier) per iteration, a block starts iteration k+1 as soon as the
+// four blocks whose rows/columns it reads -- (s, q-/+1) and (s-/+1, q) -- have published "done
+// with iteration k" (that also covers the write-after-read on the ping-pong slab).  Norm
+// iterations add one grid barrier whose last arriver reduces the partials in block order.
+// All blocks must be co-resident: the grid is sized from occupancy and the number of ranks
+// sharing the device (configure_launch).  Device mode only (host/partial modes need the host
+// between iterations).
+__global__ void __launch_bounds__(kMaxBlock + 32, 4) jacobi_persistent_kernel(const JacobiParams p, int iters) {
+  __shared__ double smem[32];
+  __shared__ int s_last;
+  extern __shared__ __align__(128) unsigned char dyn[];
+  const int NS = p.stages;
+  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
+  uint64_t* empty = full + NS;
+  float* ring = reinterpret_cast<float*>(dyn + ((32 * NS + 127) / 128) * 128);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) {
+      mbar_init(full + i, 1);
+      mbar_init(empty + i, p.consumers / 32);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  const int s = blockIdx.x % p.strips;
+  const int q = blockIdx.x / p.strips;
+  const int lane = threadIdx.x & 31;
+  const int nc = p.consumers;
+  const int x4 = (int)threadIdx.x < nc ? s * nc + (int)threadIdx.x : 0x3fffffff;
+  const bool valid = x4 < p.nx4;
+  const int lo = 1 + (int)(((long long)q * p.n) / p.chunks);
+  const int hi = (int)(((long long)(q + 1) * p.n) / p.chunks);
+  const uint64_t k0 = p.k_dev[0];
+  int ring_uses = 0;
+  for (int it = 0; it < iters; ++it) {
+    const uint64_t k = k0 + (uint64_t)it;
+    if (it > 0) {
+      if (threadIdx.x == 0) {
+        const int b = blockIdx.x;
+        if (q > 0) wait_ge(p.blk_done + (b - p.strips), k, p.timeout_ns, p.err);
+        if (q < p.chunks - 1) wait_ge(p.blk_done + (b + p.strips), k, p.timeout_ns, p.err);
+        if (s > 0) wait_ge(p.blk_done + (b - 1), k, p.timeout_ns, p.err);
+        if (s < p.strips - 1) wait_ge(p.blk_done + (b + 1), k, p.timeout_ns, p.err);
+      }
+      __syncthreads();
+    }
+    const bool do_norm = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
+    const int par = (int)(k & 1);
+    const float* src = p.slab[par];
+    float* dst = p.slab[par ^ 1];
+    double acc = 0.0;
+    int a = lo, b = hi;
+    if (q == 0) {
+      if (do_norm) boundary_row<true>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
+      else boundary_row<false>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
+    }
+    if (q == p.chunks - 1 && p.n >= 2) {
+      if (do_norm) boundary_row<true>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+      else boundary_row<false>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+    }
+    if (a < 2) a = 2;
+    if (b > p.n - 1) b = p.n - 1;
+    if (a <= b) {
+      if (do_norm)
+        ring_uses = march_staged<true>(p, src, dst, s, x4, valid, a, b, acc, ring, full, empty, ring_uses, it > 0);
+      else
+        ring_uses = march_staged<false>(p, src, dst, s, x4, valid, a, b, acc, ring, full, empty, ring_uses, it > 0);
+    }
+    __syncthreads();  // every store of this block's iteration k is issued
+    if (threadIdx.x == 0) {
+      __threadfence();
+      st_release_sys(p.blk_done + blockIdx.x, k + 1);
+    }
+    if (do_norm) {
+      const double t = block_sum(acc, smem);
+      if (threadIdx.x == 0) {
+        p.partials[blockIdx.x] = t;
+        const unsigned gen = *(volatile unsigned int*)(p.nbar + 1);
+        __threadfence();
+        s_last = atomicAdd(p.nbar, 1u) == gridDim.x - 1;
+        if (!s_last) {
+          unsigned ns = 32;
+          while (*(volatile unsigned int*)(p.nbar + 1) == gen) {
+            __nanosleep(ns);
+            if (ns < 256) ns <<= 1;
+          }
+          __threadfence();
+        }
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        double v = 0.0;
+        for (int i = threadIdx.x; i < (int)gridDim.x; i += blockDim.x) v += p.partials[i];
+        const double tot = block_sum(v, smem);
+        if (threadIdx.x == 0) {
+          norm_publish(p, tot);
+          *(volatile unsigned int*)p.nbar = 0;
+          __threadfence();
+          atomicAdd(p.nbar + 1, 1u);  // release the grid barrier
+        }
+      }
+      __syncthreads();
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(p.done, 1u) == gridDim.x - 1;
+    if (s_last) {
+      __threadfence();
+      p.k_dev[0] = k0 + (uint64_t)iters;
+      *p.done = 0;
+      __threadfence();
+    }
+  }
+}
+
+int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s) {
+  jacobi_persistent_kernel<<<grid, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p, iters);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
 }
 
 // Host mode: after ncclAllReduce of rank_sum, record sqrt into the history and bump m.
@@ -924,8 +1062,9 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
 int preload_kernels() {
   UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
   UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  UC_CUDA(cudaFuncSetAttribute(jacobi_persistent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
   const void* fns[] = {(const void*)jacobi_iter_kernel<0>, (const void*)jacobi_iter_kernel<1>,
-                       (const void*)jacobi_iter_kernel<2>,
+                       (const void*)jacobi_iter_kernel<2>, (const void*)jacobi_persistent_kernel,
                        (const void*)norm_finish_kernel,
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
@@ -940,7 +1079,9 @@ int preload_kernels() {
 }
 
 int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm) {
-  if (variant == 2)
+  if (variant == 3)
+    UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_persistent_kernel, block, smem));
+  else if (variant == 2)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<2>, block, smem));
   else if (variant == 1)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<1>, block, smem));

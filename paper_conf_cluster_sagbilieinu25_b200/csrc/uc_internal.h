@@ -54,6 +54,8 @@ struct JacobiParams {
   unsigned long long* k_dev;           // local iteration counter
   unsigned int* done;                  // local block ticket
   unsigned int* work;                  // local dynamic tile counter (variant 2)
+  unsigned int* nbar;                  // local [count, generation] norm grid barrier (variant 3)
+  uint64_t* blk_done;                  // local [grid] last iteration each block completed (variant 3)
   int tile_rows;                       // variant 2: rows per work item
   double* partials;                    // local [grid] per-block partial sums
   double* rank_sum;                    // local: this rank's sum of squares (host-mode allreduce in place)
@@ -83,6 +85,7 @@ constexpr int kDefaultTileRows = 64;
 
 // Launch wrappers implemented in kernels.cu
 int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s);
+int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
 int launch_init_field(float* slab0, float* slab1, int nx, int n, int ny, int row0, int ring,
@@ -195,6 +198,7 @@ struct uc_jacobi {
   unsigned long long* k_dev = nullptr;
   unsigned int* done = nullptr;
   double* partials = nullptr;
+  uint64_t* blk_done = nullptr;  // [partials_cap] per-block completed iteration (variant 3)
   double* rank_sum = nullptr;
   double* norm_hist = nullptr;
   int norm_cap = 4096;

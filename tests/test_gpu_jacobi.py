@@ -163,7 +163,22 @@ def test_staged_variants_shapes(nx, ny, P, variant, tile):
         _check(nx, ny, P, topology, "device", 13, norm_every=4, variant=variant, tile_rows=tile)
 
 
-@pytest.mark.parametrize("variant", [0, 1, 2])
+@pytest.mark.parametrize("P,topology,ne", [(1, "ring", 3), (1, "dirichlet", 1), (2, "ring", 5), (3, "dirichlet", 4),
+                                           (4, "ring", 0), (8, "ring", 7)])
+def test_persistent_variant(P, topology, ne):
+    """Variant 3: one launch runs all iterations, blocks synchronise with their 4 neighbours,
+    norm rounds use a grid barrier; virtual ranks share the GPU (grid sized for co-residency)."""
+    res = _check(1028, 48 * P, P, topology, "device", 23, norm_every=ne, variant=3, chunks_of_run=[1, 9, 13])
+    assert res["launch"]["variant"] == 3
+
+
+def test_persistent_variant_stepwise_and_modes():
+    _check(1028, 64, 2, "ring", "device", 6, norm_every=2, variant=3, stepwise=True)
+    _check(1028, 64, 1, "ring", "host", 9, norm_every=2, variant=3)
+    _check(1028, 64, 1, "ring", "partial", 9, norm_every=2, variant=3)
+
+
+@pytest.mark.parametrize("variant", [0, 1, 2, 3])
 def test_full_size_each_variant(variant):
     """16384^2, device mode, 3 iterations, whole grid bit-exact for every kernel variant."""
     _check(16384, 16384, 1, "ring", "device", 3, norm_every=1, variant=variant)
