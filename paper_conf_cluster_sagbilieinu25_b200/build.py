@@ -56,6 +56,8 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     sources (compile-time tuning knobs in csrc/kernels.cu), loaded with UC_LIB_PATH=<out>."""
     target = out or LIB
     if not force and not defines and out is None and not _stale():
+        if any(not os.path.exists(s[:-2]) for s in glob.glob(os.path.join(ROOT, "examples", "*.c"))):
+            build_examples()
         return LIB
     nd = nccl_dir()
     os.makedirs(os.path.dirname(os.path.abspath(target)), exist_ok=True)
@@ -74,7 +76,17 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     if verbose:
         sys.stderr.write(res.stderr)
     os.replace(tmp, target)
+    if out is None:
+        build_examples()
     return target
+
+
+def build_examples() -> None:
+    """Plain-C users of the ABI (examples/*.c), linked against the in-tree library."""
+    for src in glob.glob(os.path.join(ROOT, "examples", "*.c")):
+        exe = src[:-2]
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-I", INCLUDE, src, "-o", exe, "-L", PKG,
+                               "-l:libuniconn_b200.so", "-Wl,-rpath," + PKG])
 
 
 if __name__ == "__main__":
