@@ -413,7 +413,7 @@ __device__ __forceinline__ void march_dynamic(const JacobiParams& p, const float
         if (i >= NS) mbar_wait(empty + st, (unsigned)((i / NS) - 1) & 1u);
         hdr[st] = StageHdr{done ? -1 : y, y0, s, 0};
         if (done) {
-          mbar_arrive(full + st);  // header only, no bytes
+          mbar_arrive_expect_tx(full + st, 0);  // header only, no bytes
           return;
         }
         mbar_arrive_expect_tx(full + st, bytes);

@@ -1,0 +1,45 @@
+"""Small end-to-end runs of every kernel variant and launch mode, for compute-sanitizer:
+
+    compute-sanitizer --tool memcheck|racecheck|synccheck|initcheck python scripts/sanitize_run.py
+
+Checks each result against the oracle as well (bit-exact grid).  Sizes are tiny because the
+tools slow kernels down by orders of magnitude; spin-wait timeouts are raised accordingly.
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tests"))
+
+import numpy as np  # noqa: E402
+
+import oracle  # noqa: E402
+from gpu_harness import assert_slabs_equal_global, solve_gpu  # noqa: E402
+from inputs import gen  # noqa: E402
+
+import gpu_harness  # noqa: E402
+
+
+def main():
+    cases = [
+        dict(P=1, mode="device", variant=1), dict(P=1, mode="device", variant=0), dict(P=1, mode="device", variant=2),
+        dict(P=1, mode="device", variant=3), dict(P=1, mode="host", variant=1), dict(P=1, mode="partial", variant=1),
+        dict(P=2, mode="device", variant=1), dict(P=2, mode="device", variant=3),
+    ]
+    if len(sys.argv) > 1:
+        cases = cases[: int(sys.argv[1])]
+    nx, ny, iters, ne = 132, 24, 4, 2
+    for c in cases:
+        P = c["P"]
+        res = solve_gpu(nx, ny * P, P, "ring", c["mode"], iters, ne if c["mode"] != "partial" or P == 1 else 0,
+                        variant=c["variant"], use_graph=False)
+        want, _ = oracle.jacobi_run(gen.global_field(nx, ny * P, "ring"), iters, "ring")
+        assert_slabs_equal_global(res["final"], want, P, "ring")
+        print("ok", c, flush=True)
+    print("SANITIZE_RUN_DONE")
+
+
+if __name__ == "__main__":
+    gpu_harness.TIMEOUT_S = 300.0
+    main()

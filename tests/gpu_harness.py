@@ -8,6 +8,7 @@ from inputs import gen
 from vranks import run_ranks
 
 MODES = {"device": 1, "host": 0, "partial": 2}
+TIMEOUT_S = 5.0  # device spin-wait timeout (raised by scripts/sanitize_run.py)
 
 
 def neighbours(U, topology):
@@ -30,7 +31,7 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
         comm = U.Comm(env, top, bot)
         stream = torch.cuda.Stream()
         coord = U.Coord(comm, MODES[mode], stream.cuda_stream)
-        coord.set_timeout(5.0)
+        coord.set_timeout(TIMEOUT_S)
         J = U.Jacobi(comm, nx, ny, seed, zero_init)
         try:
             if block_x or blocks_per_sm or variant >= 0 or stages or tile_rows:
