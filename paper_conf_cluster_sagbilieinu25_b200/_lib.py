@@ -26,6 +26,7 @@ UC_MODE_HOST, UC_MODE_DEVICE, UC_MODE_PARTIAL = 0, 1, 2
 UC_F32, UC_F64, UC_U64 = 0, 1, 2
 UC_TOPO_NONE, UC_TOPO_RING, UC_TOPO_CHAIN = 0, 1, 2
 UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_P2P_HALO = 0, 1, 2
+UC_SUM, UC_PROD, UC_MIN, UC_MAX = 0, 1, 2, 3
 UC_MAX_RANKS = 8
 
 ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p)
@@ -58,6 +59,15 @@ _SIGS = {
     "uc_signal_wait": (i32, [vp, vp, sz, sz, vp, sz, u64, i32]),
     "uc_allreduce_sum": (i32, [vp, vp, vp, sz, i32]),
     "uc_p2p_bench": (i32, [vp, i32, vp, vp, sz, i32, i32, i32, i32, i32]),
+    "uc_allreduce": (i32, [vp, vp, vp, sz, i32, i32]),
+    "uc_reduce": (i32, [vp, vp, vp, sz, i32, i32, i32]),
+    "uc_broadcast": (i32, [vp, vp, sz, sz, i32]),
+    "uc_allgather": (i32, [vp, vp, vp, sz, sz]),
+    "uc_allgatherv": (i32, [vp, vp, sz, vp, sz, P(sz), P(sz)]),
+    "uc_alltoall": (i32, [vp, vp, vp, sz, sz]),
+    "uc_gather": (i32, [vp, vp, vp, sz, sz, i32]),
+    "uc_scatter": (i32, [vp, vp, vp, sz, sz, i32]),
+    "uc_coord_barrier": (i32, [vp]),
     "uc_jacobi_create": (i32, [vp, i32, i32, u64, i32, P(vp)]),
     "uc_jacobi_step": (i32, [vp, vp, i32, vp]),
     "uc_jacobi_run": (i32, [vp, vp, i32, i32, vp, i32]),

@@ -944,47 +944,68 @@ struct PeerFlags {
   uint64_t* p[UC_MAX_RANKS];
 };
 
+// ReductionOperator: SUM, PROD, MIN, MAX.  Every rank applies the operator to slots
+// 0..P-1 in rank order, so all ranks hold bit-identical results (reading G12).
 template <typename T>
-__device__ void oneshot_body(const T* send, T* recv, size_t count, int rank, int size, const PeerPtrs& slots,
-                             const PeerFlags& flags, const uint64_t* my_flags, const char* my_slots,
-                             uint64_t epoch, size_t slot_bytes, unsigned long long timeout_ns, unsigned int* err) {
+__device__ __forceinline__ T apply_op(int op, T a, T b) {
+  switch (op) {
+    case UC_PROD: return a * b;
+    case UC_MIN: return b < a ? b : a;
+    case UC_MAX: return b > a ? b : a;
+    default: return a + b;
+  }
+}
+
+// One-shot reduction over the coordinator's symmetric slots: root < 0 -> AllReduce (every rank
+// stores its vector into slot[rank] of every rank and reduces), else Reduce to `root` (only the
+// root's slots are written and only the root waits and reduces).
+template <typename T>
+__device__ void oneshot_body(const T* send, T* recv, size_t count, int rank, int size, int op, int root,
+                             const PeerPtrs& slots, const PeerFlags& flags, const uint64_t* my_flags,
+                             const char* my_slots, uint64_t epoch, size_t slot_bytes, unsigned long long timeout_ns,
+                             unsigned int* err) {
   const int par = (int)(epoch & 1);
   for (int q = 0; q < size; ++q) {
+    if (root >= 0 && q != root) continue;
     T* dst = reinterpret_cast<T*>(static_cast<char*>(slots.p[q]) + (size_t)(par * size + rank) * slot_bytes);
     for (size_t i = threadIdx.x; i < count; i += blockDim.x) dst[i] = send[i];
   }
   __syncthreads();
+  const bool receiver = root < 0 || rank == root;
   if (threadIdx.x == 0) {
     __threadfence_system();
-    for (int q = 0; q < size; ++q) st_release_sys(flags.p[q] + (size_t)(par * size + rank) * kFlagStride, epoch);
     for (int q = 0; q < size; ++q)
-      wait_ge(my_flags + (size_t)(par * size + q) * kFlagStride, epoch, timeout_ns, err);
+      if (root < 0 || q == root) st_release_sys(flags.p[q] + (size_t)(par * size + rank) * kFlagStride, epoch);
+    if (receiver)
+      for (int q = 0; q < size; ++q)
+        wait_ge(my_flags + (size_t)(par * size + q) * kFlagStride, epoch, timeout_ns, err);
   }
   __syncthreads();
+  if (!receiver) return;
   for (size_t i = threadIdx.x; i < count; i += blockDim.x) {
     T acc = T(0);
     for (int q = 0; q < size; ++q) {
       const volatile T* src =
           reinterpret_cast<const volatile T*>(my_slots + (size_t)(par * size + q) * slot_bytes);
-      acc = acc + src[i];
+      acc = q == 0 ? src[i] : apply_op<T>(op, acc, src[i]);
     }
     recv[i] = acc;
   }
 }
 
-__global__ void allreduce_oneshot_kernel(const void* send, void* recv, size_t count, int dtype, int rank, int size,
-                                         PeerPtrs slots, PeerFlags flags, const uint64_t* my_flags,
+__global__ void allreduce_oneshot_kernel(const void* send, void* recv, size_t count, int dtype, int op, int root,
+                                         int rank, int size, PeerPtrs slots, PeerFlags flags, const uint64_t* my_flags,
                                          const char* my_slots, uint64_t epoch, size_t slot_bytes,
                                          unsigned long long timeout_ns, unsigned int* err) {
   if (dtype == UC_F32)
-    oneshot_body<float>((const float*)send, (float*)recv, count, rank, size, slots, flags, my_flags, my_slots, epoch,
-                        slot_bytes, timeout_ns, err);
+    oneshot_body<float>((const float*)send, (float*)recv, count, rank, size, op, root, slots, flags, my_flags,
+                        my_slots, epoch, slot_bytes, timeout_ns, err);
   else if (dtype == UC_F64)
-    oneshot_body<double>((const double*)send, (double*)recv, count, rank, size, slots, flags, my_flags, my_slots,
-                         epoch, slot_bytes, timeout_ns, err);
+    oneshot_body<double>((const double*)send, (double*)recv, count, rank, size, op, root, slots, flags, my_flags,
+                         my_slots, epoch, slot_bytes, timeout_ns, err);
   else
-    oneshot_body<unsigned long long>((const unsigned long long*)send, (unsigned long long*)recv, count, rank, size,
-                                     slots, flags, my_flags, my_slots, epoch, slot_bytes, timeout_ns, err);
+    oneshot_body<unsigned long long>((const unsigned long long*)send, (unsigned long long*)recv, count, rank, size, op,
+                                     root, slots, flags, my_flags, my_slots, epoch, slot_bytes, timeout_ns, err);
 }
 
 // ------------------------------------------------------------------------------ launchers
@@ -1040,8 +1061,8 @@ int launch_signal_wait(const uint64_t* sig, uint64_t val, unsigned long long tim
   return UC_OK;
 }
 
-int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dtype, int rank, int size,
-                             void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
+int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dtype, int op, int root, int rank,
+                             int size, void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
                              const void* my_slots, uint64_t epoch, size_t slot_bytes, unsigned long long timeout_ns,
                              unsigned int* err, cudaStream_t s) {
   PeerPtrs sp{};
@@ -1050,7 +1071,7 @@ int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dty
     sp.p[q] = peer_slots[q];
     fp.p[q] = peer_flags[q];
   }
-  allreduce_oneshot_kernel<<<1, 256, 0, s>>>(send, recv, count, dtype, rank, size, sp, fp, my_flags,
+  allreduce_oneshot_kernel<<<1, 256, 0, s>>>(send, recv, count, dtype, op, root, rank, size, sp, fp, my_flags,
                                              (const char*)my_slots, epoch, slot_bytes, timeout_ns, err);
   UC_CUDA(cudaGetLastError());
   return UC_OK;

@@ -362,6 +362,8 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
   auto cleanup = [&](int rc) {
     if (k->err) cudaFree(k->err);
     if (k->put_counter) cudaFree(k->put_counter);
+    if (k->nccl_scratch) cudaFree(k->nccl_scratch);
+    if (k->nccl) ncclCommDestroy(k->nccl);
     delete k;
     return rc;
   };
@@ -371,6 +373,8 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
   if (e == cudaSuccess) e = cudaMalloc(&k->put_counter, 4 * sizeof(unsigned int));
   if (e == cudaSuccess) e = cudaMemset(k->put_counter, 0, 4 * sizeof(unsigned int));
   k->p2p_bar = k->put_counter + 1;
+  if (e == cudaSuccess) e = cudaMalloc(&k->nccl_scratch, sizeof(float));
+  if (e == cudaSuccess) e = cudaMemset(k->nccl_scratch, 0, sizeof(float));
   if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
   if (e != cudaSuccess) return cleanup(fail(UC_ERR_CUDA, "coordinator state: %s", cudaGetErrorString(e)));
   // host mode: NCCL for everything; partial mode: NCCL for collectives, created at the
@@ -389,6 +393,11 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
         uc_mem_free_symmetric(k->ar_scratch);
         return cleanup(fail(UC_ERR_UNSUPPORTED, "device mode needs every rank peer-addressable; rank %d is not", q));
       }
+    rc = uc_mem_alloc_symmetric(c, 2 * P * kFlagStride * sizeof(uint64_t), &k->coll_flags);
+    if (rc != UC_OK) {
+      uc_mem_free_symmetric(k->ar_scratch);
+      return cleanup(rc);
+    }
   }
   c->live_objects++;
   *out = k;
@@ -402,8 +411,10 @@ int uc_coord_destroy(uc_coord* k) {
   cudaStreamSynchronize(k->stream);
   if (k->nccl) ncclCommDestroy(k->nccl);
   if (k->ar_scratch) UC_TRY(uc_mem_free_symmetric(k->ar_scratch));
+  if (k->coll_flags) UC_TRY(uc_mem_free_symmetric(k->coll_flags));
   cudaFree(k->err);
   cudaFree(k->put_counter);
+  cudaFree(k->nccl_scratch);
   k->comm->live_objects--;
   delete k;
   return UC_OK;
@@ -582,20 +593,17 @@ int uc_p2p_bench(uc_coord* k, int pattern, uc_mem* buf, uc_mem* sig, size_t byte
 }
 
 int uc_allreduce_sum(uc_coord* k, const void* send, void* recv, size_t count, uc_dtype dt) {
-  if (!k || !send || !recv) return fail(UC_ERR_ARG, "NULL argument");
+  return uc_allreduce(k, send, recv, count, dt, UC_SUM);  // collectives.cu
+}
+
+}  // extern "C"
+
+int uc::oneshot_reduce(uc_coord* k, const void* send, void* recv, size_t count, uc_dtype dt, uc_redop op, int root) {
   if (dt != UC_F32 && dt != UC_F64 && dt != UC_U64) return fail(UC_ERR_ARG, "unknown dtype %d", (int)dt);
   uc_comm* c = k->comm;
-  UC_CUDA(cudaSetDevice(c->env->device));
-  if (count == 0) return UC_OK;
-  if (k->mode != UC_MODE_DEVICE) {  // host mode, and partial mode ("collectives as PureHost")
-    UC_TRY(ensure_nccl(k));
-    ncclDataType_t t = dt == UC_F32 ? ncclFloat32 : dt == UC_F64 ? ncclFloat64 : ncclUint64;
-    UC_NCCL(ncclAllReduce(send, recv, count, t, ncclSum, k->nccl, k->stream));
-    return UC_OK;
-  }
   const size_t esz = dt == UC_F32 ? 4 : 8;
   if (count * esz > k->ar_slot_bytes)
-    return fail(UC_ERR_UNSUPPORTED, "device-mode allreduce supports <= %zu bytes, got %zu", k->ar_slot_bytes,
+    return fail(UC_ERR_UNSUPPORTED, "device-mode reductions support <= %zu bytes, got %zu", k->ar_slot_bytes,
                 count * esz);
   const size_t P = (size_t)c->size;
   void* slots[UC_MAX_RANKS];
@@ -607,9 +615,7 @@ int uc_allreduce_sum(uc_coord* k, const void* send, void* recv, size_t count, uc
   }
   char* mine = (char*)k->ar_scratch->local;
   const uint64_t epoch = ++k->ar_epoch;
-  return launch_allreduce_oneshot(send, recv, count, (int)dt, c->rank, c->size, slots, flags,
+  return launch_allreduce_oneshot(send, recv, count, (int)dt, (int)op, root, c->rank, c->size, slots, flags,
                                   (const uint64_t*)(mine + 2 * P * k->ar_slot_bytes), mine, epoch, k->ar_slot_bytes,
                                   k->timeout_ns, k->err, k->stream);
 }
-
-}  // extern "C"

@@ -95,10 +95,12 @@ int launch_put_signal(const void* src, void* dst, size_t bytes, uint64_t* sig, u
                       unsigned int* counter, cudaStream_t s);
 int launch_signal_wait(const uint64_t* sig, uint64_t val, unsigned long long timeout_ns, unsigned int* err,
                        cudaStream_t s);
-int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dtype, int rank, int size,
-                             void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
+int launch_allreduce_oneshot(const void* send, void* recv, size_t count, int dtype, int op, int root, int rank,
+                             int size, void* const* peer_slots, uint64_t* const* peer_flags, const uint64_t* my_flags,
                              const void* my_slots, uint64_t epoch, size_t slot_bytes,
                              unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
+// device-mode one-shot AllReduce (root < 0) / Reduce (to root) over the coordinator's slots
+int oneshot_reduce(uc_coord* k, const void* send, void* recv, size_t count, uc_dtype dt, uc_redop op, int root);
 int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm);
 struct P2PLaunch {
   const void* src;
@@ -172,6 +174,9 @@ struct uc_coord {
   uc_mem* ar_scratch = nullptr;        // device-mode allreduce slots [2][P][slot_bytes] + flags
   size_t ar_slot_bytes = 32768;
   uint64_t ar_epoch = 0;
+  uc_mem* coll_flags = nullptr;        // device/partial: [ready P][done P] flags of the collectives
+  uint64_t coll_epoch = 0;
+  float* nccl_scratch = nullptr;       // host-mode barrier operand
   uint64_t p2p_epoch[3][UC_MAX_RANKS] = {};  // signal base of the next uc_p2p_bench call, per (pattern, peer)
   unsigned int* p2p_bar = nullptr;     // grid barrier [count, gen] of the p2p kernel
   int live_jacobi_users = 0;

@@ -19,7 +19,8 @@ from typing import Callable, Optional
 import numpy as np
 
 from ._lib import (ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
-                   UC_P2P_HALO, UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_TOPO_CHAIN, UC_TOPO_NONE, UC_TOPO_RING, UC_U64,
+                   UC_MAX, UC_MIN, UC_P2P_HALO, UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_PROD, UC_SUM, UC_TOPO_CHAIN,
+                   UC_TOPO_NONE, UC_TOPO_RING, UC_U64,
                    UCError, check, lib)
 
 AllgatherImpl = Callable[[bytes, int], bytes]  # (my bytes, bytes_per_rank) -> size*bytes_per_rank bytes
@@ -183,6 +184,35 @@ class Coord:
                   peer: int = 0, role: int = 0, blocks: int = 0):
         check(lib.uc_p2p_bench(self.h, pattern, buf.h, sig.h, nbytes, iters, window, peer, role, blocks),
               "uc_p2p_bench")
+
+    def allreduce(self, send: int, recv: int, count: int, dtype: int, op: int = 0):
+        check(lib.uc_allreduce(self.h, C.c_void_p(send), C.c_void_p(recv), count, dtype, op), "uc_allreduce")
+
+    def reduce(self, send: int, recv: int, count: int, dtype: int, op: int, root: int):
+        check(lib.uc_reduce(self.h, C.c_void_p(send), C.c_void_p(recv or None), count, dtype, op, root), "uc_reduce")
+
+    def broadcast(self, buf: SymMem, off: int, nbytes: int, root: int):
+        check(lib.uc_broadcast(self.h, buf.h, off, nbytes, root), "uc_broadcast")
+
+    def allgather(self, send: int, recv: SymMem, recv_off: int, nbytes: int):
+        check(lib.uc_allgather(self.h, C.c_void_p(send), recv.h, recv_off, nbytes), "uc_allgather")
+
+    def allgatherv(self, send: int, nbytes: int, recv: SymMem, recv_off: int, counts, displs):
+        n = len(counts)
+        c_arr, d_arr = (C.c_size_t * n)(*counts), (C.c_size_t * n)(*displs)
+        check(lib.uc_allgatherv(self.h, C.c_void_p(send), nbytes, recv.h, recv_off, c_arr, d_arr), "uc_allgatherv")
+
+    def alltoall(self, send: int, recv: SymMem, recv_off: int, nbytes: int):
+        check(lib.uc_alltoall(self.h, C.c_void_p(send), recv.h, recv_off, nbytes), "uc_alltoall")
+
+    def gather(self, send: int, recv: SymMem, recv_off: int, nbytes: int, root: int):
+        check(lib.uc_gather(self.h, C.c_void_p(send), recv.h, recv_off, nbytes, root), "uc_gather")
+
+    def scatter(self, send: int, recv: SymMem, recv_off: int, nbytes: int, root: int):
+        check(lib.uc_scatter(self.h, C.c_void_p(send or None), recv.h, recv_off, nbytes, root), "uc_scatter")
+
+    def barrier(self):
+        check(lib.uc_coord_barrier(self.h), "uc_coord_barrier")
 
     def allreduce_sum(self, send: int, recv: int, count: int, dtype: int):
         check(lib.uc_allreduce_sum(self.h, C.c_void_p(send), C.c_void_p(recv), count, dtype), "uc_allreduce_sum")
