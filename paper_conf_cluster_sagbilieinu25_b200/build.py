@@ -56,7 +56,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     sources (compile-time tuning knobs in csrc/kernels.cu), loaded with UC_LIB_PATH=<out>."""
     target = out or LIB
     if not force and not defines and out is None and not _stale():
-        if any(not os.path.exists(s[:-2]) for s in glob.glob(os.path.join(ROOT, "examples", "*.c"))):
+        if any(not os.path.exists(t) or os.path.getmtime(t) < os.path.getmtime(s) for s, t in _example_targets()):
             build_examples()
         return LIB
     nd = nccl_dir()
@@ -81,12 +81,24 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     return target
 
 
+def _example_targets():
+    ex = os.path.join(ROOT, "examples")
+    t = [(s, s[:-2]) for s in glob.glob(os.path.join(ex, "*.c"))]
+    t += [(s, os.path.join(ex, "lib" + os.path.basename(s)[:-3].replace("device_api_ring", "uc_device_example") + ".so"))
+          for s in glob.glob(os.path.join(ex, "*.cu"))]
+    return t
+
+
 def build_examples() -> None:
-    """Plain-C users of the ABI (examples/*.c), linked against the in-tree library."""
-    for src in glob.glob(os.path.join(ROOT, "examples", "*.c")):
-        exe = src[:-2]
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-I", INCLUDE, src, "-o", exe, "-L", PKG,
-                               "-l:libuniconn_b200.so", "-Wl,-rpath," + PKG])
+    """Users of the library: plain-C drivers of the C-ABI (examples/*.c, gcc) and user kernels
+    written against the header-only device API (examples/*.cu, nvcc sm_100a, shared library)."""
+    for src, target in _example_targets():
+        if src.endswith(".c"):
+            subprocess.check_call(["gcc", "-O2", "-std=c11", "-I", INCLUDE, src, "-o", target, "-L", PKG,
+                                   "-l:libuniconn_b200.so", "-Wl,-rpath," + PKG])
+        else:
+            subprocess.check_call([nvcc(), *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
+                                   "-I", INCLUDE, src, "-o", target])
 
 
 if __name__ == "__main__":

@@ -4,32 +4,14 @@
 #pragma once
 #include <cstdint>
 
+#include "uniconn_device.cuh"  // the public device API: signals, waits, grouped puts
+
 namespace uc {
 namespace dev {
 
-__device__ __forceinline__ unsigned long long globaltimer() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-
-__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-
-__device__ __forceinline__ uint64_t ld_relaxed_sys_u64(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-
-__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
-
-__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
-  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
+__device__ __forceinline__ unsigned long long globaltimer() { return uc_dev_globaltimer(); }
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) { return uc_dev_ld_acquire(p); }
+__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) { uc_dev_signal(p, v, UC_DEV_SIGNAL_SET); }
 
 __device__ __forceinline__ void st_relaxed_sys_f64(double* p, double v) {
   asm volatile("st.relaxed.sys.global.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
@@ -41,40 +23,15 @@ __device__ __forceinline__ double ld_relaxed_sys_f64(const double* p) {
   return v;
 }
 
-// Acknowledge / nvshmem_signal_wait_until(GE) for one thread.  Returns false on timeout (and
-// sets bit 0 of *err).  Monotone ">=" instead of the listing's "==": a neighbour one
-// iteration ahead must not hang us (reading G10).
+// Acknowledge / nvshmem_signal_wait_until(GE) for one thread (uc_dev_wait_ge).  Returns false
+// on timeout (and sets bit 0 of *err).  Monotone ">=" instead of the listing's "==": a
+// neighbour one iteration ahead must not hang us (reading G10).  Once one wait has timed out the
+// others give up at once, so a broken peer costs one timeout, not one per pending wait.
 __device__ __forceinline__ bool wait_ge(const uint64_t* flag, uint64_t v, unsigned long long timeout_ns,
                                         unsigned int* err) {
-  if (ld_acquire_sys(flag) >= v) return true;
-  unsigned long long t0 = globaltimer();
-  unsigned ns = 32;
-  // poll with relaxed loads (no L1 invalidation per poll); the fence after the observing load
-  // turns it into an acquire pattern
-  while (ld_relaxed_sys_u64(flag) < v) {
-    // give up at the timeout, or at once if an earlier wait already timed out (so a broken
-    // peer costs one timeout, not one per pending wait)
-    if (globaltimer() - t0 > timeout_ns || *(volatile unsigned int*)err) {
-      atomicOr(err, 1u);
-      return false;
-    }
-    __nanosleep(ns);
-    if (ns < 256) ns <<= 1;
-  }
-  fence_acq_rel_sys();
-  return true;
+  return uc_dev_wait_ge(flag, v, timeout_ns, err);
 }
 
-// Block-wide signal release after the block's stores (put_signal_nbi_block): every
-// thread's stores are ordered before the barrier; one thread fences at system scope and
-// release-stores the flag.
-__device__ __forceinline__ void block_signal_release(uint64_t* flag, uint64_t v) {
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence_system();
-    st_release_sys(flag, v);
-  }
-}
 
 // ---- mbarrier + bulk-copy (TMA engine) helpers, sm_90+ PTX, used by the staged y-march
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
