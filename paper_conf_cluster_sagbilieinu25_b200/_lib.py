@@ -68,6 +68,11 @@ _SIGS = {
     "uc_gather": (i32, [vp, vp, vp, sz, sz, i32]),
     "uc_scatter": (i32, [vp, vp, vp, sz, sz, i32]),
     "uc_coord_barrier": (i32, [vp]),
+    "uc_cg_create": (i32, [vp, i32, i32, i32, i32, u64, P(vp)]),
+    "uc_cg_run": (i32, [vp, vp, i32, vp, i32]),
+    "uc_cg_copy_x": (i32, [vp, vp, vp]),
+    "uc_cg_info": (i32, [vp, P(i64), P(i64), P(i64), P(i64), P(i64)]),
+    "uc_cg_destroy": (i32, [vp]),
     "uc_jacobi_create": (i32, [vp, i32, i32, u64, i32, P(vp)]),
     "uc_jacobi_step": (i32, [vp, vp, i32, vp]),
     "uc_jacobi_run": (i32, [vp, vp, i32, i32, vp, i32]),

@@ -95,6 +95,7 @@ int uc_env_init(int world_rank, int world_size, int device, uc_allgather_fn ag, 
     UC_CUDA(cudaSetDevice(device));
     UC_CUDA(cudaFree(nullptr));  // create the primary context now
     UC_TRY(preload_kernels());   // no lazy module loads once ranks spin on each other
+    UC_TRY(preload_cg_kernels());
   }
   uc_env* e = new uc_env;
   e->rank = world_rank;

@@ -121,6 +121,7 @@ int launch_wait_halo(const uint64_t* my_flags, int strips, int flag_half, int ha
                      unsigned long long timeout_ns, unsigned int* err, cudaStream_t s);
 size_t staged_smem_bytes(int consumers, int stages);
 int preload_kernels();
+int preload_cg_kernels();
 int ensure_nccl(uc_coord* k);
 const void* builtin_kernel(const char* name);
 

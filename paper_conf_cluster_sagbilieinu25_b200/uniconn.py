@@ -229,6 +229,34 @@ def builtin_kernel(name: str) -> int:
     return p.value
 
 
+class CG:
+    """The §VI-D Conjugate Gradient workload on the synthetic 3-D stencil matrix (uniconn.h)."""
+
+    def __init__(self, comm: Comm, nx: int, ny: int, nz: int, stencil: int = 27, seed: int = 0xC6):
+        h = C.c_void_p()
+        check(lib.uc_cg_create(comm.h, nx, ny, nz, stencil, seed, C.byref(h)), "uc_cg_create")
+        self.h, self.comm = h, comm
+        n, nl, r0, nnz, it = (C.c_int64() for _ in range(5))
+        check(lib.uc_cg_info(h, C.byref(n), C.byref(nl), C.byref(r0), C.byref(nnz), C.byref(it)), "uc_cg_info")
+        self.N, self.n_local, self.row0, self.nnz_local = n.value, nl.value, r0.value, nnz.value
+
+    def run(self, coord: Coord, iters: int, use_graph: bool = True,
+            rr_out: Optional[np.ndarray] = None) -> np.ndarray:
+        out = rr_out if rr_out is not None else np.zeros(iters, np.float64)
+        check(lib.uc_cg_run(coord.h, self.h, iters, C.c_void_p(out.ctypes.data), int(use_graph)), "uc_cg_run")
+        return out[:iters]
+
+    def x(self, coord: Coord) -> np.ndarray:
+        a = np.empty(self.n_local, np.float64)
+        check(lib.uc_cg_copy_x(coord.h, self.h, C.c_void_p(a.ctypes.data)), "uc_cg_copy_x")
+        return a
+
+    def destroy(self):
+        if self.h:
+            check(lib.uc_cg_destroy(self.h), "uc_cg_destroy")
+            self.h = None
+
+
 class Jacobi:
     """The §VI-C Jacobi solver on this rank's slab (see uniconn.h for layout and semantics)."""
 
