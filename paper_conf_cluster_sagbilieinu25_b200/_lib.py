@@ -2,7 +2,7 @@
 
 The library is the product: there is no Python or CPU fallback.  If the shared library is
 missing this module raises ImportError (build it with ``python -m
-paper_conf_cluster_sagbilieinu25_b200.build`` or ``__graft_entry__.build()``).
+paper_conf_cluster_sagbilieinu25_b200/build.py`` or ``__graft_entry__.build()``).
 """
 from __future__ import annotations
 
@@ -14,7 +14,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("UC_LIB_PATH") or os.path.join(_PKG, "libuniconn_b200.so")
 
 if not os.path.exists(LIB_PATH):
-    raise ImportError(f"{LIB_PATH} is missing: run `python -m paper_conf_cluster_sagbilieinu25_b200.build` "
+    raise ImportError(f"{LIB_PATH} is missing: run `python paper_conf_cluster_sagbilieinu25_b200/build.py` "
                       "(the CUDA path has no fallback)")
 
 lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
@@ -73,6 +73,7 @@ _SIGS = {
     "uc_cg_copy_x": (i32, [vp, vp, vp]),
     "uc_cg_info": (i32, [vp, P(i64), P(i64), P(i64), P(i64), P(i64)]),
     "uc_cg_destroy": (i32, [vp]),
+    "uc_cg_set_launch": (i32, [vp, i32, i32]),
     "uc_jacobi_create": (i32, [vp, i32, i32, u64, i32, P(vp)]),
     "uc_jacobi_step": (i32, [vp, vp, i32, vp]),
     "uc_jacobi_run": (i32, [vp, vp, i32, i32, vp, i32]),

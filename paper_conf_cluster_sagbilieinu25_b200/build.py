@@ -1,6 +1,8 @@
 """Build libuniconn_b200.so in-tree with nvcc for sm_100a (no torch extension machinery).
 
-    python -m paper_conf_cluster_sagbilieinu25_b200.build [--force]
+    python paper_conf_cluster_sagbilieinu25_b200/build.py [--force] [--define X=Y --out path.so]
+
+(run it as a script, not with -m: importing the package loads the library being built)
 
 The library links the NCCL shipped in the torch wheel (``nvidia/nccl``, 2.28.x) with an rpath
 to it, and CUDA's static runtime (nvcc default), so it loads beside torch in one process.

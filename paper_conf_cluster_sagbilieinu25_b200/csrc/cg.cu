@@ -108,6 +108,21 @@ __device__ bool cg_finish(const CGParams& p, double acc, double* smem, int* s_la
   return true;
 }
 
+// streaming loads of the matrix (read once per iteration; keep L1 for the gathered p)
+__device__ __forceinline__ double ld_stream_f64(const double* a) {
+  double v;
+  asm volatile("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(a));
+  return v;
+}
+__device__ __forceinline__ int ld_stream_s32(const int* a) {
+  int v;
+  asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(a));
+  return v;
+}
+
+// CSR SpMV with TPR lanes per row and U rows in flight per lane group (memory-level
+// parallelism for the dependent col -> p gathers); row sums reduced by shuffles in lane order.
+template <int TPR, int U>
 __global__ void __launch_bounds__(256) cg_spmv_kernel(const CGParams p) {
   __shared__ double smem[32];
   __shared__ int s_last;
@@ -117,20 +132,43 @@ __global__ void __launch_bounds__(256) cg_spmv_kernel(const CGParams p) {
       for (int q = 0; q < p.size; ++q) wait_ge(p.pflag_mine + (size_t)q * kFlagStride, k, p.timeout_ns, p.err);
     __syncthreads();
   }
-  const int sub = threadIdx.x % kTPR;
-  const unsigned mask = 0xffu << ((threadIdx.x & 31) & ~(kTPR - 1));
-  const long long rows_per_pass = (long long)gridDim.x * blockDim.x / kTPR;
+  const int sub = threadIdx.x % TPR;
+  const unsigned mask = (TPR == 32 ? 0xffffffffu : ((1u << TPR) - 1u)) << ((threadIdx.x & 31) & ~(TPR - 1));
+  const long long groups = (long long)gridDim.x * blockDim.x / TPR;
+  const double* __restrict__ pf = p.pfull;
   double acc = 0.0;
-  for (long long row = (blockIdx.x * (long long)blockDim.x + threadIdx.x) / kTPR; row < p.nloc;
-       row += rows_per_pass) {
-    const long long a = __ldg(p.rowptr + row), b = __ldg(p.rowptr + row + 1);
-    double s = 0.0;
-    for (long long j = a + sub; j < b; j += kTPR) s += __ldg(p.vals + j) * p.pfull[__ldg(p.cols + j)];
+  for (long long base = (blockIdx.x * (long long)blockDim.x + threadIdx.x) / TPR; base < p.nloc;
+       base += groups * U) {
+    long long a[U], b[U];
+    double s[U];
+    long long len = 0;
 #pragma unroll
-    for (int o = kTPR / 2; o > 0; o >>= 1) s += __shfl_down_sync(mask, s, o, kTPR);
-    if (sub == 0) {
-      p.q[row] = s;
-      acc += p.pfull[p.row0 + row] * s;
+    for (int u = 0; u < U; ++u) {
+      const long long row = base + u * groups;
+      a[u] = b[u] = 0;
+      if (row < p.nloc) {
+        a[u] = __ldg(p.rowptr + row);
+        b[u] = __ldg(p.rowptr + row + 1);
+      }
+      s[u] = 0.0;
+      len = max(len, b[u] - a[u]);
+    }
+    for (long long off = sub; off < len; off += TPR) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const long long j = a[u] + off;
+        if (j < b[u]) s[u] += ld_stream_f64(p.vals + j) * __ldg(pf + ld_stream_s32(p.cols + j));
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+#pragma unroll
+      for (int o = TPR / 2; o > 0; o >>= 1) s[u] += __shfl_down_sync(mask, s[u], o, TPR);
+      const long long row = base + u * groups;
+      if (sub == 0 && row < p.nloc) {
+        p.q[row] = s[u];
+        acc += pf[p.row0 + row] * s[u];
+      }
     }
   }
   double tot;
@@ -199,6 +237,24 @@ __global__ void __launch_bounds__(256) cg_pupdate_kernel(const CGParams p) {
   }
 }
 
+typedef void (*SpmvKernel)(const CGParams);
+
+template <int TPR>
+SpmvKernel spmv_for_unroll(int u) {
+  return u == 4 ? cg_spmv_kernel<TPR, 4> : u == 2 ? cg_spmv_kernel<TPR, 2> : cg_spmv_kernel<TPR, 1>;
+}
+// nullptr for unsupported (lanes_per_row in {4, 8, 16, 32}, rows_in_flight in {1, 2, 4})
+SpmvKernel spmv_kernel(int tpr, int u) {
+  if (u != 1 && u != 2 && u != 4) return nullptr;
+  switch (tpr) {
+    case 4: return spmv_for_unroll<4>(u);
+    case 8: return spmv_for_unroll<8>(u);
+    case 16: return spmv_for_unroll<16>(u);
+    case 32: return spmv_for_unroll<32>(u);
+    default: return nullptr;
+  }
+}
+
 // host/partial mode: finish alpha (which = 1) or beta/rr (which = 2) from the NCCL-reduced part
 __global__ void cg_scalar_kernel(CGState* st, double* hist, int hist_cap, int which) {
   if (which == 1) {
@@ -231,7 +287,8 @@ struct uc_cg {
   unsigned int* done = nullptr;
   double* hist = nullptr;
   int hist_cap = 65536;
-  int grid = 0;
+  int grid = 0, spmv_grid = 0, partials_cap = 0;
+  int tpr = 8, unroll = 2;  // SpMV: lanes per row, rows in flight per lane group
   long long k = 0;
   int mode = -1;  // launch mode that drives this solver (fixed after the first run)
   cudaStream_t aux = nullptr;
@@ -279,7 +336,7 @@ CGParams cg_params(const uc_coord* k, const uc_cg* cg) {
 int cg_enqueue(uc_coord* k, uc_cg* cg) {
   const CGParams p = cg_params(k, cg);
   const bool dev = k->mode == UC_MODE_DEVICE;
-  cg_spmv_kernel<<<cg->grid, 256, 0, k->stream>>>(p);
+  spmv_kernel(cg->tpr, cg->unroll)<<<cg->spmv_grid, 256, 0, k->stream>>>(p);
   UC_CUDA(cudaGetLastError());
   if (!dev) {
     UC_NCCL(ncclAllReduce(&cg->st->part, &cg->st->part, 1, ncclFloat64, ncclSum, k->nccl, k->stream));
@@ -299,6 +356,35 @@ int cg_enqueue(uc_coord* k, uc_cg* cg) {
     double* pf = (double*)cg->pfull->local;
     UC_NCCL(ncclAllGather(pf + cg->row0, pf, (size_t)cg->nloc, ncclFloat64, k->nccl, k->stream));
   }
+  return UC_OK;
+}
+
+// Launch geometry: the SpMV variant (lanes per row, rows in flight) and one wave of blocks for
+// every kernel; the block-partials buffer is sized for the larger grid.
+int cg_configure(uc_cg* cg, int tpr, int unroll) {
+  const SpmvKernel f = spmv_kernel(tpr, unroll);
+  if (!f) return fail(UC_ERR_ARG, "SpMV lanes_per_row %d (4, 8, 16, 32) / rows_in_flight %d (1, 2, 4)", tpr, unroll);
+  int sms = 148, bps = 0, bpv = 0;
+  UC_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cg->comm->env->device));
+  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, f, 256, 0));
+  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bpv, cg_update_kernel, 256, 0));
+  const long long groups_needed = (cg->nloc + unroll - 1) / unroll;
+  const int sg = (int)std::min<long long>((long long)sms * std::max(1, bps),
+                                          std::max<long long>(1, (groups_needed * tpr + 255) / 256));
+  const int vg = (int)std::min<long long>((long long)sms * std::max(1, bpv), std::max<long long>(1, (cg->nloc + 255) / 256));
+  const int need = std::max(sg, vg);
+  if (need > cg->partials_cap) {
+    if (cg->partials) cudaFree(cg->partials);
+    cg->partials = nullptr;
+    UC_CUDA(cudaMalloc(&cg->partials, sizeof(double) * need));
+    cg->partials_cap = need;
+  }
+  cg->tpr = tpr;
+  cg->unroll = unroll;
+  cg->spmv_grid = sg;
+  cg->grid = vg;
+  for (auto& g : cg->graphs) cudaGraphExecDestroy(g.exec);
+  cg->graphs.clear();
   return UC_OK;
 }
 
@@ -385,11 +471,8 @@ int uc_cg_create(uc_comm* c, int nx, int ny, int nz, int stencil, uint64_t seed,
   if (rc != UC_OK) return bail(rc);
   rc = uc_mem_alloc_symmetric(c, cg_ctrl_bytes(P), &cg->ctrl);
   if (rc != UC_OK) return bail(rc);
-  int sms = 148, bps = 0;
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->env->device);
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cg_spmv_kernel, 256, 0);
-  if (e != cudaSuccess || bps < 1) bps = 1;
-  cg->grid = (int)std::min<long long>((long long)sms * bps, std::max<long long>(1, (cg->nloc * kTPR + 255) / 256));
+  rc = cg_configure(cg, cg->tpr, cg->unroll);
+  if (rc != UC_OK) return bail(rc);
   e = cudaMalloc(&cg->rowptr, sizeof(long long) * rowptr.size());
   if (e == cudaSuccess) e = cudaMalloc(&cg->cols, sizeof(int) * std::max<size_t>(1, cols.size()));
   if (e == cudaSuccess) e = cudaMalloc(&cg->vals, sizeof(double) * std::max<size_t>(1, vals.size()));
@@ -397,7 +480,6 @@ int uc_cg_create(uc_comm* c, int nx, int ny, int nz, int stencil, uint64_t seed,
   if (e == cudaSuccess) e = cudaMalloc(&cg->r, sizeof(double) * cg->nloc);
   if (e == cudaSuccess) e = cudaMalloc(&cg->q, sizeof(double) * cg->nloc);
   if (e == cudaSuccess) e = cudaMalloc(&cg->st, sizeof(CGState));
-  if (e == cudaSuccess) e = cudaMalloc(&cg->partials, sizeof(double) * cg->grid);
   if (e == cudaSuccess) e = cudaMalloc(&cg->done, sizeof(unsigned int));
   if (e == cudaSuccess) e = cudaMalloc(&cg->hist, sizeof(double) * cg->hist_cap);
   if (e != cudaSuccess) return bail(fail(UC_ERR_OOM, "CG state: %s", cudaGetErrorString(e)));
@@ -500,6 +582,13 @@ int uc_cg_info(const uc_cg* cg, int64_t* n_global, int64_t* n_local, int64_t* ro
   return UC_OK;
 }
 
+int uc_cg_set_launch(uc_cg* cg, int lanes_per_row, int rows_in_flight) {
+  if (!cg) return fail(UC_ERR_ARG, "solver is NULL");
+  UC_CUDA(cudaSetDevice(cg->comm->env->device));
+  UC_CUDA(cudaDeviceSynchronize());
+  return cg_configure(cg, lanes_per_row > 0 ? lanes_per_row : 8, rows_in_flight > 0 ? rows_in_flight : 2);
+}
+
 int uc_cg_destroy(uc_cg* cg) {
   if (!cg) return fail(UC_ERR_ARG, "solver is NULL");
   uc_comm* c = cg->comm;
@@ -528,8 +617,10 @@ int uc_cg_destroy(uc_cg* cg) {
 
 namespace uc {
 int preload_cg_kernels() {
-  const void* fns[] = {(const void*)cg_spmv_kernel, (const void*)cg_update_kernel, (const void*)cg_pupdate_kernel,
-                       (const void*)cg_scalar_kernel};
+  std::vector<const void*> fns = {(const void*)cg_update_kernel, (const void*)cg_pupdate_kernel,
+                                  (const void*)cg_scalar_kernel};
+  for (int tpr : {4, 8, 16, 32})
+    for (int u : {1, 2, 4}) fns.push_back((const void*)spmv_kernel(tpr, u));
   for (const void* f : fns) {
     cudaFuncAttributes a;
     UC_CUDA(cudaFuncGetAttributes(&a, f));

@@ -246,6 +246,9 @@ class CG:
         check(lib.uc_cg_run(coord.h, self.h, iters, C.c_void_p(out.ctypes.data), int(use_graph)), "uc_cg_run")
         return out[:iters]
 
+    def set_launch(self, lanes_per_row: int = 0, rows_in_flight: int = 0):
+        check(lib.uc_cg_set_launch(self.h, lanes_per_row, rows_in_flight), "uc_cg_set_launch")
+
     def x(self, coord: Coord) -> np.ndarray:
         a = np.empty(self.n_local, np.float64)
         check(lib.uc_cg_copy_x(coord.h, self.h, C.c_void_p(a.ctypes.data)), "uc_cg_copy_x")

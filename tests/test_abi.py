@@ -35,6 +35,18 @@ def test_symbols_in_dynamic_table():
         assert n in syms, n
 
 
+def test_build_entry_does_not_import_the_package():
+    """__graft_entry__.build() must work on a fresh clone, where importing the package fails
+    (no library yet): the builder is loaded by file path."""
+    import subprocess
+    import sys
+    code = ("import sys, __graft_entry__ as g; b = g._builder(); "
+            "assert 'paper_conf_cluster_sagbilieinu25_b200' not in sys.modules; print(b.LIB)")
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, capture_output=True, text=True, timeout=120)
+    assert r.returncode == 0, r.stderr
+    assert r.stdout.strip().endswith("libuniconn_b200.so")
+
+
 def test_binary_is_sm100a():
     import subprocess
     out = subprocess.run(["cuobjdump", "--list-elf", U.LIB_PATH], capture_output=True, text=True).stdout
