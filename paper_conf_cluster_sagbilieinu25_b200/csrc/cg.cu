@@ -108,18 +108,6 @@ __device__ bool cg_finish(const CGParams& p, double acc, double* smem, int* s_la
   return true;
 }
 
-// streaming loads of the matrix (read once per iteration; keep L1 for the gathered p)
-__device__ __forceinline__ double ld_stream_f64(const double* a) {
-  double v;
-  asm volatile("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(a));
-  return v;
-}
-__device__ __forceinline__ int ld_stream_s32(const int* a) {
-  int v;
-  asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(a));
-  return v;
-}
-
 // CSR SpMV with TPR lanes per row and U rows in flight per lane group (memory-level
 // parallelism for the dependent col -> p gathers); row sums reduced by shuffles in lane order.
 template <int TPR, int U>
@@ -157,7 +145,9 @@ __global__ void __launch_bounds__(256) cg_spmv_kernel(const CGParams p) {
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const long long j = a[u] + off;
-        if (j < b[u]) s[u] += ld_stream_f64(p.vals + j) * __ldg(pf + ld_stream_s32(p.cols + j));
+        // read-only path with L1 allocation: a lane group's passes walk consecutive 64-byte
+        // pieces of the same 128-byte lines (no_allocate measured 40 % slower)
+        if (j < b[u]) s[u] += __ldg(p.vals + j) * __ldg(pf + __ldg(p.cols + j));
       }
     }
 #pragma unroll
@@ -288,7 +278,9 @@ struct uc_cg {
   double* hist = nullptr;
   int hist_cap = 65536;
   int grid = 0, spmv_grid = 0, partials_cap = 0;
-  int tpr = 8, unroll = 2;  // SpMV: lanes per row, rows in flight per lane group
+  // SpMV: lanes per row, rows in flight per lane group.  Round-1 sweep at 160^3, 27-point
+  // (profiles/r1_cg_sweep.txt): 4 x 2 -> 0.361 ms / iteration, 8 x 1 -> 0.45, 16 x 2 -> 0.56.
+  int tpr = 4, unroll = 2;
   long long k = 0;
   int mode = -1;  // launch mode that drives this solver (fixed after the first run)
   cudaStream_t aux = nullptr;
@@ -586,7 +578,7 @@ int uc_cg_set_launch(uc_cg* cg, int lanes_per_row, int rows_in_flight) {
   if (!cg) return fail(UC_ERR_ARG, "solver is NULL");
   UC_CUDA(cudaSetDevice(cg->comm->env->device));
   UC_CUDA(cudaDeviceSynchronize());
-  return cg_configure(cg, lanes_per_row > 0 ? lanes_per_row : 8, rows_in_flight > 0 ? rows_in_flight : 2);
+  return cg_configure(cg, lanes_per_row > 0 ? lanes_per_row : 4, rows_in_flight > 0 ? rows_in_flight : 2);
 }
 
 int uc_cg_destroy(uc_cg* cg) {
