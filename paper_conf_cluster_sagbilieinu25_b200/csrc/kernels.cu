@@ -52,6 +52,9 @@ constexpr int kPad = UC_STAGE_PAD;  // staged ring: halo floats copied on each s
 #ifndef UC_L2_EVICT_FIRST
 #define UC_L2_EVICT_FIRST 1
 #endif
+#ifndef UC_BLOCK_ORDER
+#define UC_BLOCK_ORDER 0
+#endif
 
 __device__ __forceinline__ void st4(float* p, float4 v) {
 #if UC_STORE_CS
@@ -483,8 +486,13 @@ __device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t
     march_dynamic<NORM>(p, src, dst, r0, r1, acc, ring, full, empty, hdr);
     return acc;
   }
+#if UC_BLOCK_ORDER == 1  // A/B: chunk-fastest block numbering
+  const int s = blockIdx.x / p.chunks;
+  const int q = blockIdx.x % p.chunks;
+#else  // strip-fastest: consecutive blocks sweep the same rows of adjacent strips
   const int s = blockIdx.x % p.strips;
   const int q = blockIdx.x / p.strips;
+#endif
   const int lane = threadIdx.x & 31;
   const int nc = VARIANT == 0 ? (int)blockDim.x : p.consumers;
   // the producer warp of variant 1 owns no column
