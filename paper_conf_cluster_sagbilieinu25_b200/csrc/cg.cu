@@ -141,12 +141,32 @@ __global__ void __launch_bounds__(256) cg_spmv_kernel(const CGParams p) {
       s[u] = 0.0;
       len = max(len, b[u] - a[u]);
     }
-    for (long long off = sub; off < len; off += TPR) {
+    // Rows of up to 32 nonzeros (every stencil row here) in one unrolled sweep: all the
+    // (value, column) loads first, then all the p gathers, so each lane has PASSES*U
+    // independent load chains in flight instead of one per pass.  Read-only path with L1
+    // allocation: a lane group's passes walk consecutive pieces of the same 128-byte lines
+    // (L1::no_allocate measured 40 % slower).  Longer rows fall through to the general loop.
+    constexpr int PASSES = 32 / TPR;
+    double v[PASSES][U];
+    int c[PASSES][U];
+#pragma unroll
+    for (int t = 0; t < PASSES; ++t)
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const long long j = a[u] + sub + t * TPR;
+        const bool in = j < b[u];
+        v[t][u] = in ? __ldg(p.vals + j) : 0.0;
+        c[t][u] = in ? __ldg(p.cols + j) : -1;
+      }
+#pragma unroll
+    for (int t = 0; t < PASSES; ++t)
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (c[t][u] >= 0) s[u] += v[t][u] * __ldg(pf + c[t][u]);
+    for (long long off = sub + PASSES * TPR; off < len; off += TPR) {
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const long long j = a[u] + off;
-        // read-only path with L1 allocation: a lane group's passes walk consecutive 64-byte
-        // pieces of the same 128-byte lines (no_allocate measured 40 % slower)
         if (j < b[u]) s[u] += __ldg(p.vals + j) * __ldg(pf + __ldg(p.cols + j));
       }
     }
@@ -237,6 +257,8 @@ SpmvKernel spmv_for_unroll(int u) {
 SpmvKernel spmv_kernel(int tpr, int u) {
   if (u != 1 && u != 2 && u != 4) return nullptr;
   switch (tpr) {
+    case 1: return spmv_for_unroll<1>(u);
+    case 2: return spmv_for_unroll<2>(u);
     case 4: return spmv_for_unroll<4>(u);
     case 8: return spmv_for_unroll<8>(u);
     case 16: return spmv_for_unroll<16>(u);
@@ -279,8 +301,9 @@ struct uc_cg {
   int hist_cap = 65536;
   int grid = 0, spmv_grid = 0, partials_cap = 0;
   // SpMV: lanes per row, rows in flight per lane group.  Round-1 sweep at 160^3, 27-point
-  // (profiles/r1_cg_sweep.txt): 4 x 2 -> 0.361 ms / iteration, 8 x 1 -> 0.45, 16 x 2 -> 0.56.
-  int tpr = 4, unroll = 2;
+  // (profiles/r1_cg_sweep.txt, unrolled-sweep SpMV): 4 x 1 -> 0.318 ms / iteration,
+  // 2 x 1 -> 0.370, 8 x 1 -> 0.363, 4 x 2 -> 0.355, 1 x 1 -> 0.523.
+  int tpr = 4, unroll = 1;
   long long k = 0;
   int mode = -1;  // launch mode that drives this solver (fixed after the first run)
   cudaStream_t aux = nullptr;
@@ -355,7 +378,8 @@ int cg_enqueue(uc_coord* k, uc_cg* cg) {
 // every kernel; the block-partials buffer is sized for the larger grid.
 int cg_configure(uc_cg* cg, int tpr, int unroll) {
   const SpmvKernel f = spmv_kernel(tpr, unroll);
-  if (!f) return fail(UC_ERR_ARG, "SpMV lanes_per_row %d (4, 8, 16, 32) / rows_in_flight %d (1, 2, 4)", tpr, unroll);
+  if (!f)
+    return fail(UC_ERR_ARG, "SpMV lanes_per_row %d (1, 2, 4, 8, 16, 32) / rows_in_flight %d (1, 2, 4)", tpr, unroll);
   int sms = 148, bps = 0, bpv = 0;
   UC_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cg->comm->env->device));
   UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, f, 256, 0));
@@ -578,7 +602,7 @@ int uc_cg_set_launch(uc_cg* cg, int lanes_per_row, int rows_in_flight) {
   if (!cg) return fail(UC_ERR_ARG, "solver is NULL");
   UC_CUDA(cudaSetDevice(cg->comm->env->device));
   UC_CUDA(cudaDeviceSynchronize());
-  return cg_configure(cg, lanes_per_row > 0 ? lanes_per_row : 4, rows_in_flight > 0 ? rows_in_flight : 2);
+  return cg_configure(cg, lanes_per_row > 0 ? lanes_per_row : 4, rows_in_flight > 0 ? rows_in_flight : 1);
 }
 
 int uc_cg_destroy(uc_cg* cg) {
@@ -611,7 +635,7 @@ namespace uc {
 int preload_cg_kernels() {
   std::vector<const void*> fns = {(const void*)cg_update_kernel, (const void*)cg_pupdate_kernel,
                                   (const void*)cg_scalar_kernel};
-  for (int tpr : {4, 8, 16, 32})
+  for (int tpr : {1, 2, 4, 8, 16, 32})
     for (int u : {1, 2, 4}) fns.push_back((const void*)spmv_kernel(tpr, u));
   for (const void* f : fns) {
     cudaFuncAttributes a;

@@ -87,7 +87,7 @@ def main():
     traffic = None
     if os.path.exists(rep):
         res = raw(rep)
-        lines += ["## `ncu --set full` capture of jacobi_iter_kernel", ""]
+        lines += ["## `ncu --set full` capture of the dominant kernel", ""]
         for n, d in enumerate(res):
             lines.append(f"### launch {n}: {d['Kernel Name'][:80]}")
             for m, label in METRICS:
