@@ -102,6 +102,30 @@ def rank_slab(g: np.ndarray, rank: int, size: int, topology: str = "ring") -> np
     return np.ascontiguousarray(g[rank * n: rank * n + n + 2, :])
 
 
+def rows_field(nx: int, ny: int, gys, topology: str = "ring", seed: int = DEFAULT_SEED,
+               zero_init: bool = False) -> np.ndarray:
+    """Rows of the global initial field by computed-row index gy (-1 = the top boundary/halo row,
+    NY = the bottom one; ring indices wrap), without materialising the global array."""
+    out = np.zeros((len(gys), nx), dtype=np.float32)
+    for j, gy in enumerate(gys):
+        if topology == "ring":
+            gyw = gy % ny
+            if not zero_init:
+                out[j] = interior_rows(nx, gyw, 1, seed)[0]
+            out[j, 0] = np.float32(math.sin(2.0 * math.pi * gyw / ny))
+            out[j, nx - 1] = 0.0
+        elif gy < 0:
+            out[j] = dirichlet_top_row(nx)
+        elif gy >= ny:
+            out[j] = 0.0
+        else:
+            if not zero_init:
+                out[j] = interior_rows(nx, gy, 1, seed)[0]
+            out[j, 0] = 0.0
+            out[j, nx - 1] = 0.0
+    return out
+
+
 def slab_field(nx: int, ny: int, rank: int, size: int, topology: str = "ring",
                seed: int = DEFAULT_SEED, zero_init: bool = False) -> np.ndarray:
     """Rank slab generated directly (without materialising the global array)."""

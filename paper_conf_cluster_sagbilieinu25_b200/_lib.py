@@ -81,6 +81,7 @@ _SIGS = {
     "uc_jacobi_copy_in": (i32, [vp, vp]),
     "uc_jacobi_copy_out": (i32, [vp, vp, vp, i32]),
     "uc_jacobi_copy_in_async": (i32, [vp, vp, vp]),
+    "uc_jacobi_copy_rows": (i32, [vp, vp, i32, i32, vp]),
     "uc_jacobi_copy_out_async": (i32, [vp, vp, vp]),
     "uc_jacobi_info": (i32, [vp, P(i32), P(i32), P(i32), P(i32), P(i64)]),
     "uc_jacobi_destroy": (i32, [vp]),

@@ -304,6 +304,12 @@ class Jacobi:
               "uc_jacobi_copy_out")
         return a
 
+    def copy_rows(self, coord: Optional[Coord], first_row: int, nrows: int) -> np.ndarray:
+        a = np.empty((nrows, self.nx), np.float32)
+        check(lib.uc_jacobi_copy_rows(coord.h if coord else None, self.h, first_row, nrows,
+                                      C.c_void_p(a.ctypes.data)), "uc_jacobi_copy_rows")
+        return a
+
     def copy_in_async(self, coord: Coord, host_ptr: int):
         check(lib.uc_jacobi_copy_in_async(coord.h, self.h, C.c_void_p(host_ptr)), "uc_jacobi_copy_in_async")
 

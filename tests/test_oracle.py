@@ -267,6 +267,26 @@ def test_dense_matrix_jacobi_textbook():
     assert np.abs(out[1:ny + 1, 1:nx - 1].ravel() - x).max() < 2e-6
 
 
+def test_windowed_oracle_equals_global_oracle():
+    """The sampling method of tests/test_gpu_fullsize.py: k iterations of the oracle on a window
+    of rows [y0-k-1, y1+k+1] with fixed edge rows reproduce rows y0..y1 of the global run
+    (dependency cone of k rows), including windows across the ring wrap-around."""
+    import sys, os
+    sys.path.insert(0, os.path.dirname(__file__))
+    nx, ny, k = 40, 30, 4
+    full, _ = oracle.jacobi_run(gen.global_field(nx, ny, "ring"), k, "ring")
+    for y0, y1 in ((5, 9), (-1, 3), (26, 30), (0, 0)):
+        gys = list(range(y0 - k - 1, y1 + k + 2))
+        w, _ = oracle.jacobi_run(gen.rows_field(nx, ny, gys, "ring"), k, "dirichlet")
+        got = w[k + 1:k + 1 + (y1 - y0 + 1)]
+        want = np.array([full[1 + (gy % ny)] for gy in range(y0, y1 + 1)])
+        assert np.array_equal(got, want), (y0, y1)
+    # a fixed edge row only k-1 rows away does corrupt the sample: the cone really is k rows
+    gys = list(range(5 - k + 1, 9 + k))
+    w, _ = oracle.jacobi_run(gen.rows_field(nx, ny, gys, "ring"), k, "dirichlet")
+    assert not np.array_equal(w[k - 1:k + 4], np.array([full[1 + gy] for gy in range(5, 10)]))
+
+
 def test_norm_matches_consecutive_iterates():
     """The norm record equals sum((A_{k+1}-A_k)^2) recomputed from the oracle's own grids
     (d in fp32, squares summed in double) -- north_star norm, reading G7."""
