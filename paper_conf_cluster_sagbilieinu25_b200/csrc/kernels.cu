@@ -52,6 +52,9 @@ constexpr int kPad = UC_STAGE_PAD;  // staged ring: halo floats copied on each s
 #ifndef UC_L2_EVICT_FIRST
 #define UC_L2_EVICT_FIRST 1
 #endif
+#ifndef UC_TWO_STEP_MINBLOCKS
+#define UC_TWO_STEP_MINBLOCKS 4
+#endif
 #ifndef UC_BLOCK_ORDER
 #define UC_BLOCK_ORDER 0
 #endif
@@ -179,17 +182,28 @@ __device__ __forceinline__ void march(const float* __restrict__ src, float* __re
 // bot_side: row y == n goes to the bottom neighbour's halo row 0.  Both when n == 1.
 // PartialDevice mode (device_mode == 2, Listing 6): the same puts without waits or
 // signals; the host-side Acknowledge after the kernel synchronises the neighbours.
+// Wait until the halo-row flags of strips s-1, s, s+1 on one side reach v.  The flag of strip s
+// says both "the neighbour's strip-s halo data of A_v is here" and "the neighbour's block of
+// strip s has finished reading the halo row we are about to overwrite"; the two-iteration
+// kernel (variant 4) also reads one column across each strip edge, so a writer or reader of
+// strip s waits for the adjacent strips' flags too.
+__device__ __forceinline__ void wait_strip_flags(const JacobiParams& p, int base, int s, uint64_t v) {
+  const int s0 = s > 0 ? s - 1 : 0;
+  const int s1 = s + 1 < p.strips ? s + 1 : s;
+  for (int j = s0; j <= s1; ++j) wait_ge(p.my_flags + (size_t)(base + j) * kFlagStride, v, p.timeout_ns, p.err);
+}
+
 template <bool NORM>
 __device__ __forceinline__ void boundary_row(const JacobiParams& p, const float* src, float* dst, int y, int x4,
-                                             int lane, int s, uint64_t k, bool top_side, bool bot_side,
+                                             int lane, int s, uint64_t k, int np, bool top_side, bool bot_side,
                                              double& acc) {
   const bool put_top = top_side && p.has_top;
   const bool put_bot = bot_side && p.has_bot;
   const bool fused = p.device_mode == 1;
   if (threadIdx.x == 0 && fused) {
-    // halo rows of A_k (slab k&1) must hold the neighbours' A_k rows: wait for flag >= k
-    if (put_top) wait_ge(p.my_flags + (size_t)s * kFlagStride, k, p.timeout_ns, p.err);
-    if (put_bot) wait_ge(p.my_flags + (size_t)(p.flag_half + s) * kFlagStride, k, p.timeout_ns, p.err);
+    // halo rows of A_k must hold the neighbours' A_k rows: wait for flag >= k
+    if (put_top) wait_strip_flags(p, 0, s, k);
+    if (put_bot) wait_strip_flags(p, p.flag_half, s, k);
   }
   __syncthreads();
   const bool valid = x4 < p.nx4;
@@ -199,7 +213,6 @@ __device__ __forceinline__ void boundary_row(const JacobiParams& p, const float*
   const float4 dn = ld4_co(src + (size_t)(y + 1) * pitch, x4, valid);
   const float e = ld_edge_co(src + (size_t)y * pitch, x4, lane, p.nx4, valid);
   const float4 o = row_update(up, cur, dn, e, lane, x4, p.nx4);
-  const int np = (int)((k + 1) & 1);
   if (valid) {
     reinterpret_cast<float4*>(dst + (size_t)y * pitch)[x4] = o;
     // one-sided puts straight into the neighbours' halo rows of A_{k+1} over NVLink
@@ -258,7 +271,9 @@ __device__ void norm_publish(const JacobiParams& p, double tot) {
 }
 
 // Last block: deterministic sum of the block partials, cross-rank norm (device mode), counter bumps.
-__device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* smem) {
+// advance = iterations done by this launch (2 for the two-iteration kernel, which also flips
+// the slab parity offset k_dev[2]).
+__device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* smem, int advance) {
   double tot = 0.0;
   if (do_norm) {
     double v = 0.0;
@@ -267,7 +282,8 @@ __device__ void finish_iteration(const JacobiParams& p, bool do_norm, double* sm
   }
   if (threadIdx.x == 0) {
     if (do_norm) norm_publish(p, tot);
-    p.k_dev[0] = p.k_dev[0] + 1;
+    p.k_dev[0] = p.k_dev[0] + (unsigned long long)advance;
+    if (advance == 2) p.k_dev[2] = p.k_dev[2] ^ 1ull;
     *p.done = 0;
     *p.work = 0;  // variant 2 tile counter
     __threadfence();
@@ -461,9 +477,8 @@ __device__ __forceinline__ void march_dynamic(const JacobiParams& p, const float
 
 // ------------------------------------------------------------------------------ the kernel
 template <int VARIANT, bool NORM>
-__device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t k, float* ring, uint64_t* full,
-                                                 uint64_t* empty, StageHdr* hdr) {
-  const int par = (int)(k & 1);
+__device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t k, int par, float* ring,
+                                                 uint64_t* full, uint64_t* empty, StageHdr* hdr) {
   const float* src = p.slab[par];
   float* dst = p.slab[par ^ 1];
   if (VARIANT == 2) {
@@ -477,8 +492,8 @@ __device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t
       for (int j = blockIdx.x; j < nb; j += gridDim.x) {
         const int s = j % p.strips;
         const int x4 = (int)threadIdx.x < nc ? s * nc + (int)threadIdx.x : 0x3fffffff;
-        if (j < p.strips) boundary_row<NORM>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
-        else boundary_row<NORM>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+        if (j < p.strips) boundary_row<NORM>(p, src, dst, 1, x4, lane, s, k, par ^ 1, true, p.n == 1, acc);
+        else boundary_row<NORM>(p, src, dst, p.n, x4, lane, s, k, par ^ 1, false, true, acc);
       }
       r0 = 2;
       r1 = p.n - 1;
@@ -503,8 +518,8 @@ __device__ __forceinline__ double iteration_body(const JacobiParams& p, uint64_t
   double acc = 0.0;
   int a = lo, b = hi;
   if (p.device_mode) {
-    if (q == 0) boundary_row<NORM>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
-    if (q == p.chunks - 1 && p.n >= 2) boundary_row<NORM>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+    if (q == 0) boundary_row<NORM>(p, src, dst, 1, x4, lane, s, k, par ^ 1, true, p.n == 1, acc);
+    if (q == p.chunks - 1 && p.n >= 2) boundary_row<NORM>(p, src, dst, p.n, x4, lane, s, k, par ^ 1, false, true, acc);
     if (a < 2) a = 2;
     if (b > p.n - 1) b = p.n - 1;
   }
@@ -539,13 +554,14 @@ __global__ void __launch_bounds__(kMaxBlock + 32, UC_MINBLOCKS) jacobi_iter_kern
     __syncthreads();
   }
   const uint64_t k = p.k_dev[0];
+  const int par = (int)((k + p.k_dev[2]) & 1);  // slab holding A_k (k_dev[2]: two-iteration launches so far, mod 2)
   const bool do_norm = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
   if (do_norm) {
-    const double acc = iteration_body<VARIANT, true>(p, k, ring, full, empty, hdr);
+    const double acc = iteration_body<VARIANT, true>(p, k, par, ring, full, empty, hdr);
     const double t = block_sum(acc, smem);
     if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
   } else {
-    iteration_body<VARIANT, false>(p, k, ring, full, empty, hdr);
+    iteration_body<VARIANT, false>(p, k, par, ring, full, empty, hdr);
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -556,7 +572,7 @@ __global__ void __launch_bounds__(kMaxBlock + 32, UC_MINBLOCKS) jacobi_iter_kern
   __syncthreads();
   if (s_last) {
     __threadfence();
-    finish_iteration(p, do_norm, smem);
+    finish_iteration(p, do_norm, smem, 1);
   }
 }
 
@@ -596,6 +612,7 @@ __global__ void __launch_bounds__(kMaxBlock + 32, 4) jacobi_persistent_kernel(co
   const int lo = 1 + (int)(((long long)q * p.n) / p.chunks);
   const int hi = (int)(((long long)(q + 1) * p.n) / p.chunks);
   const uint64_t k0 = p.k_dev[0];
+  const uint64_t flip = p.k_dev[2];
   int ring_uses = 0;
   for (int it = 0; it < iters; ++it) {
     const uint64_t k = k0 + (uint64_t)it;
@@ -610,18 +627,18 @@ __global__ void __launch_bounds__(kMaxBlock + 32, 4) jacobi_persistent_kernel(co
       __syncthreads();
     }
     const bool do_norm = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
-    const int par = (int)(k & 1);
+    const int par = (int)((k + flip) & 1);
     const float* src = p.slab[par];
     float* dst = p.slab[par ^ 1];
     double acc = 0.0;
     int a = lo, b = hi;
     if (q == 0) {
-      if (do_norm) boundary_row<true>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
-      else boundary_row<false>(p, src, dst, 1, x4, lane, s, k, true, p.n == 1, acc);
+      if (do_norm) boundary_row<true>(p, src, dst, 1, x4, lane, s, k, par ^ 1, true, p.n == 1, acc);
+      else boundary_row<false>(p, src, dst, 1, x4, lane, s, k, par ^ 1, true, p.n == 1, acc);
     }
     if (q == p.chunks - 1 && p.n >= 2) {
-      if (do_norm) boundary_row<true>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
-      else boundary_row<false>(p, src, dst, p.n, x4, lane, s, k, false, true, acc);
+      if (do_norm) boundary_row<true>(p, src, dst, p.n, x4, lane, s, k, par ^ 1, false, true, acc);
+      else boundary_row<false>(p, src, dst, p.n, x4, lane, s, k, par ^ 1, false, true, acc);
     }
     if (a < 2) a = 2;
     if (b > p.n - 1) b = p.n - 1;
@@ -683,6 +700,272 @@ __global__ void __launch_bounds__(kMaxBlock + 32, 4) jacobi_persistent_kernel(co
 
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s) {
   jacobi_persistent_kernel<<<grid, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p, iters);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+// ------------------------------------------------------------------------------ two iterations per launch
+// Variant 4: one launch advances A_k -> A_{k+2} (temporal blocking of depth 2).  The staged
+// y-march keeps two levels in registers: from the A_k rows r-2, r-1, r streamed through the TMA
+// ring it computes the A_{k+1} row r-1, and from the A_{k+1} rows r-3, r-2, r-1 the A_{k+2}
+// row r-2, which is the only one stored.  A_{k+1} never goes to HBM, so a launch moves 8 bytes
+// per point for two iterations.  Every iteration's boundary rows are still exchanged with
+// the neighbours (Listing 3), in two rounds per launch:
+//   prologue  (first/last row-chunk blocks of each strip, at launch start): wait for the
+//             A_k halo rows (slab flags >= k), compute the A_{k+1} rows 1 / n and put them into
+//             the neighbours' h1 rows, release their h1 flags = k+1;
+//   march     rows 2..n-1 of A_{k+2} (A_{k+1} rows 1..n recomputed on the fly);
+//   deferred  (same blocks, after their march): wait for the neighbours' A_{k+1} rows
+//             (h1 flags >= k+1), compute the A_{k+2} rows 1 / n, store them locally and into
+//             the neighbours' halo rows of the output slab, release slab flags = k+2.
+// The prologue's puts overlap the whole interior sweep; the deferred wait is exposed only by
+// the skew between neighbour launches.  Bitwise, every A_{k+1} and A_{k+2} value is the same
+// expression of the same operands as in the one-iteration kernel (same rounding, no FMA).
+// A_{k+2} goes to the other slab (A_k is still being read by other blocks), so a launch flips
+// the slab parity offset k_dev[2]: A_k lives in slab (k + k_dev[2]) & 1 for every kernel.
+
+// A_{k+1} at (y, x) from A_k read directly (boundary work; coherent loads).
+__device__ __forceinline__ float level1_point(const float* src, int y, int x, int nx) {
+  const float* r = src + (size_t)y * nx;
+  if (x == 0 || x == nx - 1) return r[x];  // fixed columns
+  return upd(r[x - 1], r[x + 1], r[x - nx], r[x + nx]);
+}
+
+// A_{k+1} row y for this thread's 4 columns (all 32 lanes must call: shuffles); c = A_k row y.
+__device__ __forceinline__ float4 level1_row(const JacobiParams& p, const float* src, int y, int x4, int lane,
+                                             bool valid, float4& c) {
+  const size_t pitch = (size_t)p.nx;
+  const float4 up = ld4_co(src + (size_t)(y - 1) * pitch, x4, valid);
+  c = ld4_co(src + (size_t)y * pitch, x4, valid);
+  const float4 dn = ld4_co(src + (size_t)(y + 1) * pitch, x4, valid);
+  const float e = ld_edge_co(src + (size_t)y * pitch, x4, lane, p.nx4, valid);
+  return row_update(up, c, dn, e, lane, x4, p.nx4);
+}
+
+// Prologue of one side: A_{k+1} boundary row (top: row 1, bottom: row n) -> neighbour's h1 row.
+template <bool N1>
+__device__ __forceinline__ void two_step_prologue(const JacobiParams& p, const float* src, int x4, int lane, int s,
+                                                  uint64_t k, bool top, double& acc) {
+  const bool has = top ? p.has_top : p.has_bot;
+  if (threadIdx.x == 0 && has) wait_strip_flags(p, top ? 0 : p.flag_half, s, k);  // A_k halo rows
+  __syncthreads();
+  const bool valid = x4 < p.nx4;
+  float4 c;
+  const float4 o = level1_row(p, src, top ? 1 : p.n, x4, lane, valid, c);
+  if (N1 && valid) acc_sq(acc, o, c);
+  if (has) {
+    // top side: our row 1 is the top neighbour's "from bottom" h1 row; bottom side: our row n is
+    // the bottom neighbour's "from top" h1 row
+    if (valid) reinterpret_cast<float4*>(top ? p.top_h1_rows + p.nx : p.bot_h1_rows)[x4] = o;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence_system();
+      if (top) st_release_sys(p.top_h1_flags + (size_t)(p.flag_half + s) * kFlagStride, k + 1);
+      else st_release_sys(p.bot_h1_flags + (size_t)s * kFlagStride, k + 1);
+    }
+  }
+}
+
+// Deferred step of one side: A_{k+2} boundary row from the A_{k+1} rows around it (the one
+// beyond the slab comes from the neighbour's prologue, or is the fixed row of a chain end).
+template <bool N2>
+__device__ __forceinline__ void two_step_deferred(const JacobiParams& p, const float* src, float* dst, int np,
+                                                  int x4, int lane, int s, uint64_t k, bool top, double& acc) {
+  const bool has = top ? p.has_top : p.has_bot;
+  if (threadIdx.x == 0 && has)
+    wait_ge(p.h1_flags + (size_t)((top ? 0 : p.flag_half) + s) * kFlagStride, k + 1, p.timeout_ns, p.err);
+  __syncthreads();
+  const bool valid = x4 < p.nx4;
+  const size_t pitch = (size_t)p.nx;
+  const int y = top ? 1 : p.n;       // the A_{k+2} row
+  const int yi = top ? 2 : p.n - 1;  // its inner A_{k+1} neighbour
+  float4 c, ci;
+  const float4 l1 = level1_row(p, src, y, x4, lane, valid, c);
+  const float4 l1i = level1_row(p, src, yi, x4, lane, valid, ci);
+  // the outer A_{k+1} row: the neighbour's, or the fixed halo row (unchanged by iterations)
+  const float* outer = has ? (top ? p.h1_rows : p.h1_rows + pitch) : src + (size_t)(top ? 0 : p.n + 1) * pitch;
+  const float4 l1o = ld4_co(outer, x4, valid);
+  // across the warp edge: lane 0 needs A_{k+1}(y, 4*x4-1), lane 31 A_{k+1}(y, 4*x4+4)
+  float e = 0.f;
+  if (valid) {
+    if (lane == 0 && x4 > 0) e = level1_point(src, y, 4 * x4 - 1, p.nx);
+    else if (lane == 31 && x4 + 1 < p.nx4) e = level1_point(src, y, 4 * x4 + 4, p.nx);
+  }
+  const float4 o = top ? row_update(l1o, l1, l1i, e, lane, x4, p.nx4) : row_update(l1i, l1, l1o, e, lane, x4, p.nx4);
+  if (N2 && valid) acc_sq(acc, o, l1);
+  if (valid) {
+    reinterpret_cast<float4*>(dst + (size_t)y * pitch)[x4] = o;
+    if (has) {
+      if (top) reinterpret_cast<float4*>(p.top_slab[np] + (size_t)(p.n + 1) * pitch)[x4] = o;
+      else reinterpret_cast<float4*>(p.bot_slab[np])[x4] = o;
+    }
+  }
+  if (has) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence_system();
+      if (top) st_release_sys(p.top_flags + (size_t)(p.flag_half + s) * kFlagStride, k + 2);  // top's from_bottom[s]
+      else st_release_sys(p.bot_flags + (size_t)s * kFlagStride, k + 2);                     // bottom's from_top[s]
+    }
+  }
+}
+
+// The two-level staged y-march: A_{k+2} rows a..b (2 <= a, b <= n-1) of strip s.  The producer
+// warp streams the A_k rows a-2..b+2; consumers keep A_k rows r-2, r-1, r and A_{k+1} rows
+// r-3, r-2, r-1 in registers.  Lanes 0 / 31 also carry the two A_k values across the warp edge
+// (ring pad) and compute the one A_{k+1} value across it, so no cross-warp exchange is needed.
+// N1: norm of iteration k (A_{k+1} - A_k over rows a..b); N2: of iteration k+1.
+template <bool N1, bool N2>
+__device__ __forceinline__ void march_two_step(const JacobiParams& p, const float* src, float* dst, int s, int x4,
+                                               bool valid, int a, int b, double& acc, float* ring, uint64_t* full,
+                                               uint64_t* empty, bool proxy_fence) {
+  const int nc = p.consumers, NS = p.stages;
+  const int ST = 4 * nc + 2 * kPad;
+  const int lane = threadIdx.x & 31;
+  const size_t pitch = (size_t)p.nx;
+  const int rows = b - a + 5;  // A_k rows a-2 .. b+2
+  if ((int)threadIdx.x >= nc) {
+    if (lane == 0) {
+      const int x0 = s * 4 * nc;
+      const int left = x0 >= kPad ? x0 - kPad : 0;
+      const int right = min(x0 + 4 * nc + kPad, p.nx);
+      const unsigned bytes = (unsigned)(right - left) * 4u;
+      const int off = left - (x0 - kPad);
+#if UC_L2_EVICT_FIRST
+      const uint64_t pol = policy_evict_first();
+#else
+      const uint64_t pol = policy_evict_normal();
+#endif
+      // halo rows were written by a peer's generic stores (acquired by thread 0 before the
+      // block barrier): order them before the TMA reads
+      if (proxy_fence) fence_proxy_async_global();
+      for (int i = 0; i < rows; ++i) {
+        const int st = i % NS;
+        if (i >= NS) mbar_wait(empty + st, (unsigned)((i / NS) - 1) & 1u);
+        mbar_arrive_expect_tx(full + st, bytes);
+        bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(a - 2 + i) * pitch + left, bytes, full + st, pol);
+      }
+    }
+    return;
+  }
+  const int t = threadIdx.x;
+  const bool l31 = lane == 31;
+  float4 u0 = make_float4(0.f, 0.f, 0.f, 0.f), u1 = u0;  // A_k rows r-2, r-1
+  float f0 = 0.f, f1 = 0.f, g1 = 0.f;                      // A_k across the edge: (r-2, +-1), (r-1, +-1), (r-1, +-2)
+  float4 w0 = u0, w1 = u0;                                 // A_{k+1} rows r-3, r-2
+  float x1 = 0.f;                                          // A_{k+1} (r-2) across the edge
+  for (int i = 0; i < rows; ++i) {
+    const int st = i % NS;
+    mbar_wait(full + st, (unsigned)(i / NS) & 1u);
+    const float* row = ring + (size_t)st * ST + kPad + 4 * t;
+    const float4 v = *reinterpret_cast<const float4*>(row);
+    float e1 = 0.f, e2 = 0.f;
+    if (lane == 0) {
+      e1 = row[-1];
+      e2 = row[-2];
+    } else if (l31) {
+      e1 = row[4];
+      e2 = row[5];
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty + st);
+    const int r = a - 2 + i;
+    if (i >= 2) {
+      // A_{k+1} row r-1
+      const float4 w2 = row_update(u0, u1, v, f1, lane, x4, p.nx4);
+      // A_{k+1}(r-1) across the warp edge: same operands as the neighbour lane's own value
+      const float xx = upd(g1, l31 ? u1.w : u1.x, f0, e1);
+      if (N1 && valid && r - 1 >= a && r - 1 <= b) acc_sq(acc, w2, u1);
+      if (i >= 4) {
+        // A_{k+2} row r-2
+        const float4 o = row_update(w0, w1, w2, x1, lane, x4, p.nx4);
+        if (valid) st4(dst + (size_t)(r - 2) * pitch + 4 * (size_t)x4, o);
+        if (N2 && valid) acc_sq(acc, o, w1);
+      }
+      w0 = w1;
+      w1 = w2;
+      x1 = xx;
+    }
+    u0 = u1;
+    u1 = v;
+    f0 = f1;
+    f1 = e1;
+    g1 = e2;
+  }
+}
+
+template <bool N1, bool N2>
+__device__ __forceinline__ double two_step_body(const JacobiParams& p, uint64_t k, int par, float* ring,
+                                                uint64_t* full, uint64_t* empty) {
+  const float* src = p.slab[par];
+  float* dst = p.slab[par ^ 1];
+  const int s = blockIdx.x % p.strips;
+  const int q = blockIdx.x / p.strips;
+  const int lane = threadIdx.x & 31;
+  const int nc = p.consumers;
+  const int x4 = (int)threadIdx.x < nc ? s * nc + (int)threadIdx.x : 0x3fffffff;
+  const bool valid = x4 < p.nx4;
+  const int lo = 1 + (int)(((long long)q * p.n) / p.chunks);
+  const int hi = (int)(((long long)(q + 1) * p.n) / p.chunks);
+  const bool top_blk = q == 0, bot_blk = q == p.chunks - 1;
+  double acc = 0.0;
+  if (top_blk) two_step_prologue<N1>(p, src, x4, lane, s, k, true, acc);
+  if (bot_blk) two_step_prologue<N1>(p, src, x4, lane, s, k, false, acc);
+  const int a = lo < 2 ? 2 : lo;
+  const int b = hi > p.n - 1 ? p.n - 1 : hi;
+  if (a <= b) march_two_step<N1, N2>(p, src, dst, s, x4, valid, a, b, acc, ring, full, empty, top_blk || bot_blk);
+  if (top_blk || bot_blk) {
+    __syncthreads();
+    if (top_blk) two_step_deferred<N2>(p, src, dst, par ^ 1, x4, lane, s, k, true, acc);
+    if (bot_blk) two_step_deferred<N2>(p, src, dst, par ^ 1, x4, lane, s, k, false, acc);
+  }
+  return acc;
+}
+
+// Device mode only, n >= 2, every row chunk >= 2 rows (configure_launch), norm_every != 1.
+__global__ void __launch_bounds__(kMaxBlock + 32, UC_TWO_STEP_MINBLOCKS) jacobi_two_step_kernel(const JacobiParams p) {
+  __shared__ double smem[32];
+  __shared__ int s_last;
+  extern __shared__ __align__(128) unsigned char dyn[];
+  const int NS = p.stages;
+  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
+  uint64_t* empty = full + NS;
+  float* ring = reinterpret_cast<float*>(dyn + ((32 * NS + 127) / 128) * 128);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) {
+      mbar_init(full + i, 1);
+      mbar_init(empty + i, p.consumers / 32);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  const uint64_t k = p.k_dev[0];
+  const int par = (int)((k + p.k_dev[2]) & 1);
+  const bool n1 = p.norm_every > 0 && (k % (uint64_t)p.norm_every) == 0;
+  const bool n2 = p.norm_every > 0 && ((k + 1) % (uint64_t)p.norm_every) == 0;
+  if (n1 || n2) {
+    const double acc = n1 ? two_step_body<true, false>(p, k, par, ring, full, empty)
+                          : two_step_body<false, true>(p, k, par, ring, full, empty);
+    const double t = block_sum(acc, smem);
+    if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
+  } else {
+    two_step_body<false, false>(p, k, par, ring, full, empty);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned t = atomicAdd(p.done, 1u);
+    s_last = (t == gridDim.x - 1);
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    finish_iteration(p, n1 || n2, smem, 2);
+  }
+}
+
+int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStream_t s) {
+  jacobi_two_step_kernel<<<grid, block, staged_smem_bytes(p.consumers, p.stages), s>>>(p);
   UC_CUDA(cudaGetLastError());
   return UC_OK;
 }
@@ -1092,9 +1375,10 @@ int preload_kernels() {
   UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
   UC_CUDA(cudaFuncSetAttribute(jacobi_iter_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
   UC_CUDA(cudaFuncSetAttribute(jacobi_persistent_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  UC_CUDA(cudaFuncSetAttribute(jacobi_two_step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
   const void* fns[] = {(const void*)jacobi_iter_kernel<0>, (const void*)jacobi_iter_kernel<1>,
                        (const void*)jacobi_iter_kernel<2>, (const void*)jacobi_persistent_kernel,
-                       (const void*)norm_finish_kernel,
+                       (const void*)jacobi_two_step_kernel, (const void*)norm_finish_kernel,
                        (const void*)init_field_kernel,  (const void*)put_signal_kernel,
                        (const void*)signal_wait_kernel, (const void*)allreduce_oneshot_kernel,
                        (const void*)wait_halo_kernel,   (const void*)p2p_bench_kernel,
@@ -1110,6 +1394,8 @@ int preload_kernels() {
 int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm) {
   if (variant == 3)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_persistent_kernel, block, smem));
+  else if (variant == 4)
+    UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_two_step_kernel, block, smem));
   else if (variant == 2)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<2>, block, smem));
   else if (variant == 1)

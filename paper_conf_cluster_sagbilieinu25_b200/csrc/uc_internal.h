@@ -49,9 +49,18 @@ struct JacobiParams {
   uint64_t* my_flags;      // local: [0, S) from_top[s], [S, 2S) from_bottom[s] (stride kFlagStride)
   uint64_t* top_flags;     // top neighbour's flag array (we set its from_bottom[s])
   uint64_t* bot_flags;     // bottom neighbour's flag array (we set its from_top[s])
+  // variant 4 (two iterations per launch): the A_{k+1} boundary rows travel through a second,
+  // small symmetric buffer per rank: rows [2][nx] (0 = from top, 1 = from bottom) and per-strip
+  // flags [2][flag_half] (from_top[s], from_bottom[s]; value k+1 = "A_{k+1} row present")
+  float* h1_rows;          // local
+  uint64_t* h1_flags;      // local
+  float* top_h1_rows;      // top neighbour's (we write its "from bottom" row)
+  uint64_t* top_h1_flags;
+  float* bot_h1_rows;      // bottom neighbour's (we write its "from top" row)
+  uint64_t* bot_h1_flags;
   double* norm_slot[UC_MAX_RANKS];     // rank q's norm slots: [2][P] doubles
   uint64_t* norm_flag[UC_MAX_RANKS];   // rank q's norm flags: [2][P] u64 (stride kFlagStride)
-  unsigned long long* k_dev;           // local iteration counter
+  unsigned long long* k_dev;           // local [k, norm round m, slab parity offset, -]
   unsigned int* done;                  // local block ticket
   unsigned int* work;                  // local dynamic tile counter (variant 2)
   unsigned int* nbar;                  // local [count, generation] norm grid barrier (variant 3)
@@ -85,6 +94,7 @@ constexpr int kDefaultTileRows = 64;
 
 // Launch wrappers implemented in kernels.cu
 int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s);
+int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
@@ -184,7 +194,7 @@ struct uc_coord {
 };
 
 struct JacobiGraph {
-  int iters = 0, norm_every = 0, parity = 0, mode = -1;
+  int iters = 0, norm_every = 0, parity = 0, flip = 0, mode = -1;
   cudaStream_t stream = nullptr;
   cudaGraphExec_t exec = nullptr;
 };
@@ -197,6 +207,8 @@ struct uc_jacobi {
   int64_t m = 0;                 // host mirror of the device norm-round counter k_dev[1]
   uc_mem* slabs = nullptr;       // symmetric: 2 * (n+2) * nx floats
   uc_mem* ctrl = nullptr;        // symmetric: flags + norm slots
+  uc_mem* h1 = nullptr;          // symmetric: A_{k+1} boundary rows + flags (variant 4)
+  int flip = 0;                  // host mirror of k_dev[2]: A_k lives in slab (k + flip) & 1
   size_t slab_elems = 0;
   int strips = 0;               // current column strips (launch geometry)
   int max_strips = 0;           // flag capacity per side = ceil(nx/4 / 32)
