@@ -58,7 +58,9 @@ def parse():
                          "ranks time-slice the GPU, so the numbers are not a benchmark)")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
     ap.add_argument("--cpu-sample-iters", type=int, default=3)
-    ap.add_argument("--variant", type=int, default=-1, help="0 register march, 1 TMA-staged (-1: library default)")
+    ap.add_argument("--variant", type=int, default=-1,
+                    help="0 register march, 1 TMA-staged, 2 dynamic tiles, 3 persistent, 4 two iterations per "
+                         "launch (-1: library default = 4)")
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--block-x", type=int, default=0)
@@ -104,14 +106,14 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def ncu_traffic(nx, n):
-    """Per-launch DRAM bytes of jacobi_iter_kernel from the committed ncu --set full summary."""
+def ncu_traffic(nx, n, kernel="jacobi_iter_kernel"):
+    """Per-launch DRAM bytes of the kernel from the committed ncu --set full summary."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
         return None
     with open(p) as f:
         d = json.load(f)
-    e = d.get(f"{nx}x{n}")
+    e = d.get(f"{kernel}:{nx}x{n}") or (d.get(f"{nx}x{n}") if kernel == "jacobi_iter_kernel" else None)
     return None if e is None else float(e["dram_bytes_per_launch"])
 
 
@@ -225,37 +227,58 @@ def run_ours(a):
     ms_per_step = t_max / a.steps
     total_pts = pts_rank * world * ips * a.steps
     glups = total_pts / (t_max / 1e3) / 1e9
-    launches = a.steps * ips + (a.steps * ((ips + a.norm_every - 1) // a.norm_every) if a.mode == "host" else 0)
+    # two-iteration launches (variant 4, device mode, n >= 2, norm_every != 1) + an odd remainder
+    two = launch_info["variant"] == 4 and a.mode == "device" and n >= 2 and a.norm_every != 1
+    per_launch = 2 if two else 1
+    launches_per_step = ips // 2 + ips % 2 if two else ips
+    launches = a.steps * launches_per_step + (
+        a.steps * ((ips + a.norm_every - 1) // a.norm_every) if a.mode == "host" else 0)
 
-    # ---------------- dominant kernel: per-launch events around single iterations (no norm / norm)
-    def kernel_ms(compute_norm, reps):
+    # ---------------- dominant kernel: per-launch events around single launches (no norm / norm)
+    def kernel_ms(compute_norm, reps, iters_per_launch):
         es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
-        buf = np.zeros(1, np.float64)
+        buf = np.zeros(2, np.float64)
         for s, e in es:
             s.record(stream)
-            J.step(coord, compute_norm, buf if compute_norm else None)
+            if iters_per_launch == 2:  # one two-iteration launch (norm_every 2: one norm round in it)
+                J.run(coord, 2, 2 if compute_norm else 0, False, norms_out=buf if compute_norm else None)
+            else:
+                J.step(coord, compute_norm, buf if compute_norm else None)
             e.record(stream)
         coord.sync()
         return statistics.mean(s.elapsed_time(e) for s, e in es)
 
     barrier(dist)
-    k_plain = allreduce_max(dist, kernel_ms(False, 50))
-    k_norm = allreduce_max(dist, kernel_ms(True, 10))
-    # the timed steps have 1 norm iteration per norm_every
+    k_plain = allreduce_max(dist, kernel_ms(False, 50, per_launch))
+    k_norm = allreduce_max(dist, kernel_ms(True, 10, per_launch))
+    # the timed steps have 1 norm round per norm_every iterations
     nn = max(1, a.norm_every) if a.norm_every > 0 else ips
-    k_avg = (k_plain * (nn - 1) + k_norm) / nn
+    nn_launches = max(1, nn // per_launch)
+    k_avg = (k_plain * (nn_launches - 1) + k_norm) / nn_launches
     peak, peak_src = measured_peaks()
+    # algorithmic bytes per launch: every point of A_k read once, every point of the launch's
+    # last iterate written once -- 8 B per point per launch, for 1 or 2 iterations
     alg_bytes = 8.0 * pts_rank
     achieved = alg_bytes / (k_plain / 1e3) / 1e9
-    roof = {"bound": "hbm", "kernel": "jacobi_iter_kernel", "achieved": round(achieved, 1), "peak": peak,
-            "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": ncu_traffic(nx, n),
-            "alg_bytes_per_launch": alg_bytes, "kernel_ms": round(k_plain, 5), "kernel_norm_ms": round(k_norm, 5),
-            "kernel_share_of_step": round(k_avg * ips / ms_per_step, 4), "peak_source": peak_src}
+    kname = "jacobi_two_step_kernel" if two else "jacobi_iter_kernel"
+    roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
+            "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": ncu_traffic(nx, n, kname),
+            "alg_bytes_per_launch": alg_bytes, "iterations_per_launch": per_launch,
+            "hbm_bytes_per_point_iteration": 8.0 / per_launch,
+            "kernel_ms": round(k_plain, 5), "kernel_norm_ms": round(k_norm, 5),
+            "kernel_share_of_step": round(k_avg * launches_per_step / ms_per_step, 4), "peak_source": peak_src}
+    if two:
+        # the one-iteration kernel in the same geometry, for comparison (8 B per point per iteration)
+        k1 = allreduce_max(dist, kernel_ms(False, 30, 1))
+        roof["one_iteration_kernel"] = {"kernel": "jacobi_iter_kernel", "kernel_ms": round(k1, 5),
+                                        "achieved": round(alg_bytes / (k1 / 1e3) / 1e9, 1),
+                                        "glups": round(pts_rank * world / (k1 / 1e3) / 1e9, 1)}
 
     # ---------------- halo exchange overlap (differential, §8 d): same slab, no neighbours
     halo = None
     if not a.no_extras:
-        halo = halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_plain)
+        halo = halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_plain, per_launch,
+                            launch_info)
 
     # ---------------- e2e through the C-ABI with pinned host buffers
     e2e = None
@@ -315,7 +338,7 @@ def run_ours(a):
         dist.destroy_process_group()
 
 
-def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full):
+def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full, per_launch, launch_info):
     """hidden = clamp(1 - (T_full - T_compute) / T_xchg, 0, 1) (SURVEY §8 d).  T_compute: the same
     slab and kernel with no neighbours (chain-less comm: top = bottom = -1 is not a valid Jacobi
     topology for P > 1, so we time a P = 1 dirichlet-chain solver of the same n rows in its own
@@ -326,10 +349,14 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
     st = torch.cuda.Stream()
     co1 = U.Coord(comm1, mode, st.cuda_stream)
     J1 = U.Jacobi(comm1, nx, n)
+    J1.set_launch(launch_info["variant"], 0, 0, launch_info["stages"])
     es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(30)]
     for s, e in es:
         s.record(st)
-        J1.step(co1, False, None)
+        if per_launch == 2:
+            J1.run(co1, 2, 0, False)
+        else:
+            J1.step(co1, False, None)
         e.record(st)
     co1.sync()
     t_comp = statistics.mean(s.elapsed_time(e) for s, e in es[5:])
@@ -357,7 +384,8 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
         co.signal_wait(row, nx * 4, nx * 4, sig, 16, i, comm.top)
     x1.record(st2)
     co.sync()
-    t_x = x0.elapsed_time(x1) / reps
+    # a two-iteration launch exchanges two rounds of boundary rows
+    t_x = x0.elapsed_time(x1) / reps * per_launch
     comm.barrier()
     row.free()
     sig.free()
@@ -369,7 +397,8 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
     hidden = max(0.0, min(1.0, 1.0 - (t_full - t_comp) / t_x)) if t_x > 0 else None
     return {"hidden_fraction": None if hidden is None else round(hidden, 4), "t_full_ms": round(t_full, 5),
             "t_compute_ms": round(t_comp, 5), "t_xchg_ms": round(t_x, 5),
-            "note": "per-iteration; t_xchg = standalone put_signal of both boundary rows + waits"}
+            "note": f"per launch ({per_launch} iteration(s)); t_xchg = standalone put_signal of both boundary "
+                    f"rows + waits, x{per_launch} rounds"}
 
 
 def cpu_baseline(nx, ny, iters):

@@ -52,8 +52,14 @@ constexpr int kPad = UC_STAGE_PAD;  // staged ring: halo floats copied on each s
 #ifndef UC_L2_EVICT_FIRST
 #define UC_L2_EVICT_FIRST 1
 #endif
+// two-iteration kernel: steady-state loop unroll and min blocks per SM (register cap 72 at 3);
+// sweep in profiles/r1_two_step_sweep.txt
+#ifndef UC_TWO_STEP_UNROLL
+#define UC_TWO_STEP_UNROLL 2
+#endif
+constexpr int kTwoStepUnroll = UC_TWO_STEP_UNROLL;
 #ifndef UC_TWO_STEP_MINBLOCKS
-#define UC_TWO_STEP_MINBLOCKS 4
+#define UC_TWO_STEP_MINBLOCKS 3
 #endif
 #ifndef UC_BLOCK_ORDER
 #define UC_BLOCK_ORDER 0
@@ -324,12 +330,18 @@ __device__ __forceinline__ int march_staged(const JacobiParams& p, const float* 
       // rows written by generic-proxy stores earlier in this launch (persistent kernel) must be
       // ordered before the async-proxy (TMA) reads
       if (proxy_fence) fence_proxy_async_global();
+      // ring use counter g = i0 + i continues across the iterations of a launch; stage and
+      // round parity are tracked incrementally (no integer division per row)
+      int st = i0 % NS;
+      unsigned ph = (unsigned)(i0 / NS) & 1u;
       for (int i = 0; i < rows; ++i) {
-        const int g = i0 + i;  // ring use counter (continues across the iterations of a launch)
-        const int st = g % NS;
-        if (g >= NS) mbar_wait(empty + st, (unsigned)((g / NS) - 1) & 1u);
+        if (i0 + i >= NS) mbar_wait(empty + st, ph ^ 1u);
         mbar_arrive_expect_tx(full + st, bytes);
         bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(y0 - 1 + i) * pitch + left, bytes, full + st, pol);
+        if (++st == NS) {
+          st = 0;
+          ph ^= 1u;
+        }
       }
     }
     return i0 + rows;
@@ -338,10 +350,10 @@ __device__ __forceinline__ int march_staged(const JacobiParams& p, const float* 
   const int t = threadIdx.x;
   float4 up = make_float4(0.f, 0.f, 0.f, 0.f), cur = up;
   float ec = 0.f;
+  int st = i0 % NS;
+  unsigned ph = (unsigned)(i0 / NS) & 1u;
   for (int i = 0; i < rows; ++i) {
-    const int g = i0 + i;
-    const int st = g % NS;
-    mbar_wait(full + st, (unsigned)(g / NS) & 1u);
+    mbar_wait(full + st, ph);
     const float* row = ring + (size_t)st * ST + kPad + 4 * t;
     const float4 v = *reinterpret_cast<const float4*>(row);
     float e = 0.f;
@@ -349,6 +361,10 @@ __device__ __forceinline__ int march_staged(const JacobiParams& p, const float* 
     else if (lane == 31) e = row[4];
     __syncwarp();
     if (lane == 0) mbar_arrive(empty + st);
+    if (++st == NS) {
+      st = 0;
+      ph ^= 1u;
+    }
     if (i == 0) {
       up = v;
     } else if (i == 1) {
@@ -815,6 +831,30 @@ __device__ __forceinline__ void two_step_deferred(const JacobiParams& p, const f
 // r-3, r-2, r-1 in registers.  Lanes 0 / 31 also carry the two A_k values across the warp edge
 // (ring pad) and compute the one A_{k+1} value across it, so no cross-warp exchange is needed.
 // N1: norm of iteration k (A_{k+1} - A_k over rows a..b); N2: of iteration k+1.
+// Consumer side of the two-level march: the next staged A_k row (own float4 + the two values
+// across the warp edge: lane 0 gets columns -1, -2, lane 31 columns +4, +5; branch-free, every
+// lane loads a float2), then release the stage.  Stage and phase advance incrementally.
+struct RingCursor {
+  int st;
+  unsigned ph;
+};
+__device__ __forceinline__ void ring_fetch(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
+                                           int t, int lane, RingCursor& c, float4& v, float& e1, float& e2) {
+  mbar_wait(full + c.st, c.ph);
+  const float* row = ring + (size_t)c.st * ST + kPad + 4 * t;
+  v = *reinterpret_cast<const float4*>(row);
+  const bool l31 = lane == 31;
+  const float2 ee = *reinterpret_cast<const float2*>(row + (l31 ? 4 : -2));
+  __syncwarp();
+  if (lane == 0) mbar_arrive(empty + c.st);
+  if (++c.st == NS) {
+    c.st = 0;
+    c.ph ^= 1u;
+  }
+  e1 = l31 ? ee.x : ee.y;
+  e2 = l31 ? ee.y : ee.x;
+}
+
 template <bool N1, bool N2>
 __device__ __forceinline__ void march_two_step(const JacobiParams& p, const float* src, float* dst, int s, int x4,
                                                bool valid, int a, int b, double& acc, float* ring, uint64_t* full,
@@ -839,58 +879,57 @@ __device__ __forceinline__ void march_two_step(const JacobiParams& p, const floa
       // halo rows were written by a peer's generic stores (acquired by thread 0 before the
       // block barrier): order them before the TMA reads
       if (proxy_fence) fence_proxy_async_global();
+      int st = 0;
+      unsigned ph = 0;
       for (int i = 0; i < rows; ++i) {
-        const int st = i % NS;
-        if (i >= NS) mbar_wait(empty + st, (unsigned)((i / NS) - 1) & 1u);
+        if (i >= NS) mbar_wait(empty + st, ph ^ 1u);
         mbar_arrive_expect_tx(full + st, bytes);
         bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(a - 2 + i) * pitch + left, bytes, full + st, pol);
+        if (++st == NS) {
+          st = 0;
+          ph ^= 1u;
+        }
       }
     }
     return;
   }
   const int t = threadIdx.x;
   const bool l31 = lane == 31;
-  float4 u0 = make_float4(0.f, 0.f, 0.f, 0.f), u1 = u0;  // A_k rows r-2, r-1
-  float f0 = 0.f, f1 = 0.f, g1 = 0.f;                      // A_k across the edge: (r-2, +-1), (r-1, +-1), (r-1, +-2)
-  float4 w0 = u0, w1 = u0;                                 // A_{k+1} rows r-3, r-2
-  float x1 = 0.f;                                          // A_{k+1} (r-2) across the edge
-  for (int i = 0; i < rows; ++i) {
-    const int st = i % NS;
-    mbar_wait(full + st, (unsigned)(i / NS) & 1u);
-    const float* row = ring + (size_t)st * ST + kPad + 4 * t;
-    const float4 v = *reinterpret_cast<const float4*>(row);
-    float e1 = 0.f, e2 = 0.f;
-    if (lane == 0) {
-      e1 = row[-1];
-      e2 = row[-2];
-    } else if (l31) {
-      e1 = row[4];
-      e2 = row[5];
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty + st);
-    const int r = a - 2 + i;
-    if (i >= 2) {
-      // A_{k+1} row r-1
-      const float4 w2 = row_update(u0, u1, v, f1, lane, x4, p.nx4);
-      // A_{k+1}(r-1) across the warp edge: same operands as the neighbour lane's own value
-      const float xx = upd(g1, l31 ? u1.w : u1.x, f0, e1);
-      if (N1 && valid && r - 1 >= a && r - 1 <= b) acc_sq(acc, w2, u1);
-      if (i >= 4) {
-        // A_{k+2} row r-2
-        const float4 o = row_update(w0, w1, w2, x1, lane, x4, p.nx4);
-        if (valid) st4(dst + (size_t)(r - 2) * pitch + 4 * (size_t)x4, o);
-        if (N2 && valid) acc_sq(acc, o, w1);
-      }
-      w0 = w1;
-      w1 = w2;
-      x1 = xx;
-    }
-    u0 = u1;
-    u1 = v;
-    f0 = f1;
-    f1 = e1;
-    g1 = e2;
+  const int nx4 = p.nx4;
+  RingCursor cur{0, 0u};
+  // Names: u0, u1 = A_k rows r-2, r-1 (v = row r, just fetched); f0, f1 = A_k across the warp
+  // edge (+-1 column) of rows r-2, r-1, g1 = (+-2 columns) of row r-1; w0, w1 = A_{k+1} rows
+  // r-3, r-2 and x1 = A_{k+1}(r-2) across the edge.  A_{k+1} across the edge is computed from the
+  // same operands as the neighbouring lane's own value, so it is bit-identical to it.
+  float4 u0, u1, v, w0, w1;
+  float f0, f1, g1, e1, e2, x1;
+  // rows a-2, a-1
+  ring_fetch(ring, full, empty, ST, NS, t, lane, cur, u0, f0, e2);
+  ring_fetch(ring, full, empty, ST, NS, t, lane, cur, u1, f1, g1);
+  // row a: A_{k+1} row a-1 (outside this block's rows: no norm term)
+  ring_fetch(ring, full, empty, ST, NS, t, lane, cur, v, e1, e2);
+  w0 = row_update(u0, u1, v, f1, lane, x4, nx4);  // its value across the edge is not needed
+  u0 = u1, u1 = v, f0 = f1, f1 = e1, g1 = e2;
+  // row a+1: A_{k+1} row a
+  ring_fetch(ring, full, empty, ST, NS, t, lane, cur, v, e1, e2);
+  w1 = row_update(u0, u1, v, f1, lane, x4, nx4);
+  x1 = upd(g1, l31 ? u1.w : u1.x, f0, e1);
+  if (N1 && valid) acc_sq(acc, w1, u1);
+  u0 = u1, u1 = v, f0 = f1, f1 = e1, g1 = e2;
+  // steady state: fetch row r = y+2, A_{k+1} row y+1, A_{k+2} row y, for y = a..b
+  float* out = dst + (size_t)a * pitch + 4 * (size_t)x4;
+#pragma unroll(kTwoStepUnroll)
+  for (int y = a; y <= b; ++y) {
+    ring_fetch(ring, full, empty, ST, NS, t, lane, cur, v, e1, e2);
+    const float4 w2 = row_update(u0, u1, v, f1, lane, x4, nx4);
+    const float xx = upd(g1, l31 ? u1.w : u1.x, f0, e1);
+    if (N1 && valid && y < b) acc_sq(acc, w2, u1);
+    const float4 o = row_update(w0, w1, w2, x1, lane, x4, nx4);
+    if (valid) st4(out, o);
+    if (N2 && valid) acc_sq(acc, o, w1);
+    out += pitch;
+    w0 = w1, w1 = w2, x1 = xx;
+    u0 = u1, u1 = v, f0 = f1, f1 = e1, g1 = e2;
   }
 }
 

@@ -86,10 +86,13 @@ struct JacobiParams {
 };
 
 constexpr int kFlagStride = 16;  // u64 per flag = 128 bytes, one flag per L2 line
-// Defaults from the round-1 sweep at 16384^2 (profiles/r1_sweep.txt): the TMA-staged march
-// with a 3-row ring reaches 6.36 TB/s vs 6.07 for the register march; deeper rings lose.
-constexpr int kDefaultVariant = 1;
+// Defaults from the round-1 sweeps at 16384^2 (profiles/r1_sweep.txt, r1_two_step_sweep.txt):
+// the TMA-staged march with a 3-row ring reaches 6.36 TB/s vs 6.07 for the register march
+// (deeper rings lose); the two-iteration kernel (variant 4, 3 blocks/SM, 4-row ring) moves the
+// same 8 B/point per launch at 6.4 TB/s for two iterations, so it is the default.
+constexpr int kDefaultVariant = 4;
 constexpr int kDefaultStages = 3;
+constexpr int kDefaultStagesTwoStep = 4;
 constexpr int kDefaultTileRows = 64;
 
 // Launch wrappers implemented in kernels.cu

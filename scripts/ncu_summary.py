@@ -31,6 +31,7 @@ METRICS = [
     ("sm__cycles_active.avg", "SM active cycles"),
     ("sm__cycles_elapsed.avg", "SM elapsed cycles"),
     ("smsp__inst_executed.sum", "warp instructions"),
+    ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue slots busy %"),
     ("sm__cycles_elapsed.avg.per_second", "SM clock"),
 ]
 

@@ -27,7 +27,8 @@ def window_oracle(nx, ny, y0, y1, k, topology="ring"):
     return out[k + 1:k + 1 + (y1 - y0 + 1)]
 
 
-def test_weak_scaling_8x16384sq_sampled_rows():
+@pytest.mark.parametrize("variant", [4, 1])
+def test_weak_scaling_8x16384sq_sampled_rows(variant):
     import torch
 
     import paper_conf_cluster_sagbilieinu25_b200 as U
@@ -42,6 +43,8 @@ def test_weak_scaling_8x16384sq_sampled_rows():
         co = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
         co.set_timeout(30.0)
         J = U.Jacobi(comm, nx, ny)
+        if variant != 4:
+            J.set_launch(variant)
         try:
             comm.barrier()
             J.run(co, k, 2, use_graph=True)
@@ -59,7 +62,7 @@ def test_weak_scaling_8x16384sq_sampled_rows():
             env.finalize()
 
     res = run_ranks(P, body)
-    assert res[0][3]["variant"] == 1
+    assert res[0][3]["variant"] == variant
     for r in range(P):
         top, bot, mid, _ = res[r]
         g0 = r * n  # global computed row of slab row 1

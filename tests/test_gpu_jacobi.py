@@ -71,9 +71,10 @@ def test_ragged_random_boundaries(nx):
 
 @pytest.mark.parametrize("P", [2, 3, 4, 8])
 @pytest.mark.parametrize("topology", ["ring", "dirichlet"])
-def test_partition_invariance_device_mode(P, topology):
+@pytest.mark.parametrize("variant", [1, 4])
+def test_partition_invariance_device_mode(P, topology, variant):
     """Virtual ranks: P = 2..8 give the oracle's global grid bit for bit (invariant 6)."""
-    _check(520, 24 * P, P, topology, "device", 25, norm_every=5)
+    _check(520, 24 * P, P, topology, "device", 25, norm_every=5, variant=variant)
 
 
 @pytest.mark.parametrize("P,ny", [(2, 2), (4, 4), (3, 3), (2, 4)])
@@ -178,7 +179,7 @@ def test_persistent_variant_stepwise_and_modes():
     _check(1028, 64, 1, "ring", "partial", 9, norm_every=2, variant=3)
 
 
-@pytest.mark.parametrize("variant", [0, 1, 2, 3])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
 def test_full_size_each_variant(variant):
     """16384^2, device mode, 3 iterations, whole grid bit-exact for every kernel variant."""
     _check(16384, 16384, 1, "ring", "device", 3, norm_every=1, variant=variant)
@@ -265,27 +266,33 @@ def test_constant_field_fixed_and_zero_norm():
 # --------------------------------------------------------------------------- full size
 def test_full_size_16384_single_gpu_bench_configuration():
     """BASELINE.json configs[2]/[3] at P = 1 (16384^2 fp32, 1 GiB per slab), in the launch
-    configuration bench.py times (device mode, ring, CUDA graph, default geometry): the whole
-    grid bit-exact vs the oracle after 6 iterations, norms within 1e-5."""
-    _check(16384, 16384, 1, "ring", "device", 6, norm_every=3)
+    configuration bench.py times (device mode, ring, CUDA graph, default geometry = variant 4,
+    two iterations per launch): the whole grid bit-exact vs the oracle after 6 and 7 iterations
+    (odd: a one-iteration launch at the end), norms within 1e-5 on both levels."""
+    res = _check(16384, 16384, 1, "ring", "device", 6, norm_every=3)
+    assert res["launch"]["variant"] == 4 and res["launch"]["stages"] == 4
+    _check(16384, 16384, 1, "ring", "device", 7, norm_every=2)
 
 
 def test_full_size_host_mode():
     _check(16384, 16384, 1, "ring", "host", 2, norm_every=1)
 
 
-def test_config1_4096_2ranks_1000_iterations():
+@pytest.mark.parametrize("variant", [1, 4])
+def test_config1_4096_2ranks_1000_iterations(variant):
     """BASELINE.json configs[1]: 4096 x 4096, 1000 iterations, row-split over 2 ranks, device
     put-signal (virtual ranks on one GPU), norm every 100: whole grid bit-exact."""
-    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100)
+    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, variant=variant)
 
 
-def test_config2_strong_16384_over_8_ranks():
-    """BASELINE.json configs[2] at P = 8 (2048 rows per rank), norm allreduce every iteration
-    here (every 100 in the benchmark): whole grid bit-exact after 4 iterations."""
-    _check(16384, 16384, 8, "ring", "device", 4, norm_every=2)
+@pytest.mark.parametrize("variant", [1, 4])
+def test_config2_strong_16384_over_8_ranks(variant):
+    """BASELINE.json configs[2] at P = 8 (2048 rows per rank), norm allreduce every other
+    iteration here (every 100 in the benchmark): whole grid bit-exact after 4 iterations."""
+    _check(16384, 16384, 8, "ring", "device", 4, norm_every=2, variant=variant)
 
 
-def test_config3_weak_16384_per_rank_2_ranks():
+@pytest.mark.parametrize("variant", [1, 4])
+def test_config3_weak_16384_per_rank_2_ranks(variant):
     """BASELINE.json configs[3] at P = 2: 16384 x 32768 global, 16384 x 16384 per rank."""
-    _check(16384, 32768, 2, "ring", "device", 3, norm_every=1)
+    _check(16384, 32768, 2, "ring", "device", 4, norm_every=3, variant=variant)

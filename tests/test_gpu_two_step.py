@@ -172,17 +172,3 @@ def test_subnormal_front_no_ftz():
         s = res["final"][0]
         want = np.float32(2.0 ** (-2 * k)) if k <= 74 else np.float32(0.0)
         assert s[1, k] == want and s[1, k + 1] == 0.0
-
-
-def test_full_size_16384():
-    """16384^2 (configs[2]/[3] at P = 1) in the geometry bench.py --variant 4 times: whole grid
-    bit-exact after 6 iterations (3 launches), norms at both levels."""
-    _check(16384, 16384, 1, "ring", "device", 6, norm_every=3, variant=4)
-
-
-def test_config2_strong_16384_over_8_ranks():
-    _check(16384, 16384, 8, "ring", "device", 4, norm_every=2, variant=4)
-
-
-def test_config1_4096_2ranks_1000_iterations():
-    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, variant=4)
