@@ -86,6 +86,11 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
   return p;
 }
 
+// Barrier among the first `count` threads of the block (count a multiple of 32), id 1..15.
+__device__ __forceinline__ void named_barrier_sync(int id, int count) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+
 // splitmix64 finaliser (Steele, Lea, Flood 2014) -- the input recipe's counter-based generator.
 __device__ __forceinline__ uint64_t splitmix64(uint64_t x) {
   uint64_t z = x + 0x9E3779B97F4A7C15ull;

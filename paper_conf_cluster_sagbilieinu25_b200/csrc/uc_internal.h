@@ -66,6 +66,8 @@ struct JacobiParams {
   unsigned int* nbar;                  // local [count, generation] norm grid barrier (variant 3)
   uint64_t* blk_done;                  // local [grid] last iteration each block completed (variant 3)
   int tile_rows;                       // variant 2: rows per work item
+  int strip4;                          // variant 5: owned float4 columns per strip (ghost-lane layout)
+  int chunk_shrink;                    // variant 5: rows taken off the first/last row chunk
   double* partials;                    // local [grid] per-block partial sums
   double* rank_sum;                    // local: this rank's sum of squares (host-mode allreduce in place)
   double* norm_hist;                   // local: norms by round m (ring of norm_cap)
@@ -98,6 +100,7 @@ constexpr int kDefaultTileRows = 64;
 // Launch wrappers implemented in kernels.cu
 int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStream_t s);
+int launch_jacobi_t(const JacobiParams& p, int grid, int block, int T, cudaStream_t s);
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
@@ -212,6 +215,9 @@ struct uc_jacobi {
   uc_mem* ctrl = nullptr;        // symmetric: flags + norm slots
   uc_mem* h1 = nullptr;          // symmetric: A_{k+1} boundary rows + flags (variant 4)
   int flip = 0;                  // host mirror of k_dev[2]: A_k lives in slab (k + flip) & 1
+  int levels = 1;                // variant 5: iterations per launch T
+  int strip4 = 0;                // variant 5: owned float4 columns per strip
+  int chunk_shrink = 0;          // variant 5: rows taken off the first/last row chunk
   size_t slab_elems = 0;
   int strips = 0;               // current column strips (launch geometry)
   int max_strips = 0;           // flag capacity per side = ceil(nx/4 / 32)

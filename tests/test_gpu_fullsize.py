@@ -27,7 +27,7 @@ def window_oracle(nx, ny, y0, y1, k, topology="ring"):
     return out[k + 1:k + 1 + (y1 - y0 + 1)]
 
 
-@pytest.mark.parametrize("variant", [4, 1])
+@pytest.mark.parametrize("variant", [4, 1, 5])
 def test_weak_scaling_8x16384sq_sampled_rows(variant):
     import torch
 
@@ -44,7 +44,7 @@ def test_weak_scaling_8x16384sq_sampled_rows(variant):
         co.set_timeout(30.0)
         J = U.Jacobi(comm, nx, ny)
         if variant != 4:
-            J.set_launch(variant)
+            J.set_launch(variant)  # variant 5: T = 4 iterations per launch (k = 4: one launch)
         try:
             comm.barrier()
             J.run(co, k, 2, use_graph=True)

@@ -1,0 +1,178 @@
+"""GPU parity of kernel variant 5 (T = 1..4 Jacobi iterations per launch, temporal blocking of
+depth T, ghost-lane layout) against the CPU oracle.
+
+Variant 5 keeps A_{k+1}..A_{k+T-1} in registers and stores only A_{k+T}; the boundary rows of
+every intermediate iterate are still exchanged with the neighbours (rounds 1..T per launch).
+The bar is the north_star's: the grid bit-exact after N iterations, norms within 1e-5.  Counts
+that are not multiples of T, norm cadences below T and thin slabs fall back to shorter launches
+of the same layout; every mixture must stay bit-exact.
+"""
+import numpy as np
+import pytest
+
+from gpu_harness import assert_slabs_equal_global, bits, solve_gpu
+from test_gpu_jacobi import NORM_RTOL, _check, _oracle
+
+pytestmark = pytest.mark.gpu
+
+TS = [1, 2, 3, 4]
+
+
+def _v5(T, **kw):
+    return dict(variant=5, tile_rows=T, **kw)
+
+
+@pytest.mark.parametrize("T", TS)
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+@pytest.mark.parametrize("iters,ne", [(100, 10), (101, 10), (37, 3), (40, 0)])
+def test_c1_256(T, topology, iters, ne):
+    """configs[0] (256^2, 100 iterations, 1 GPU); odd counts and norm cadences below T."""
+    res = _check(256, 256, 1, topology, "device", iters, norm_every=ne, **_v5(T))
+    assert res["launch"]["variant"] == 5 and res["launch"]["tile_rows"] == T
+
+
+@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("nx,ny,iters", [(4, 8, 9), (8, 9, 20), (12, 16, 9), (1028, 64, 38), (2052, 33, 13),
+                                         (4096, 40, 8), (36, 8, 12), (40, 9, 11), (964, 30, 17)])
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+def test_shapes_single_rank(T, nx, ny, iters, topology):
+    """Ragged strips (NX/4 not a multiple of 30 owned lanes), tiny grids, thin slabs."""
+    _check(nx, ny, 1, topology, "device", iters, norm_every=4, **_v5(T))
+
+
+@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+def test_partition_invariance(T, P, topology):
+    """Virtual ranks P = 2..8: every intermediate level's edge rows cross ranks (h buffers)."""
+    _check(520, 24 * P, P, topology, "device", 27, norm_every=5, **_v5(T))
+
+
+@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("P,ny", [(2, 4), (2, 6), (3, 9), (2, 8), (4, 32), (2, 16)])
+def test_few_rows_per_rank(T, P, ny):
+    """n = 2..8: launches shrink to the deepest T' with n >= 2T'; one row chunk per strip."""
+    for topology in ("ring", "dirichlet"):
+        _check(64, ny, P, topology, "device", 13, norm_every=0, **_v5(T))
+
+
+@pytest.mark.parametrize("T", [2, 4])
+@pytest.mark.parametrize("block_x,bps,stages", [(32, 1, 3), (64, 2, 4), (128, 0, 2), (256, 1, 8), (96, 0, 5)])
+def test_launch_geometries(T, block_x, bps, stages):
+    """Strip width (ghost lanes meet strip edges), chunk count and ring depth: 4 ranks."""
+    res = _check(1028, 128, 4, "ring", "device", 12, norm_every=4, block_x=block_x, blocks_per_sm=bps,
+                 stages=stages, **_v5(T))
+    assert res["launch"]["variant"] == 5
+
+
+@pytest.mark.parametrize("T", [2, 3, 4])
+def test_random_values_everywhere(T):
+    nx, ny = 1028, 48
+    rng = np.random.default_rng(11)
+    init = rng.random((ny + 2, nx), dtype=np.float32)
+    init[0], init[-1] = init[ny], init[1]
+    _check(nx, ny, 1, "ring", "device", 14, norm_every=7, init=init, **_v5(T))
+    _check(nx, ny, 3, "ring", "device", 14, norm_every=4, init=init, **_v5(T))
+    _check(nx, ny, 2, "dirichlet", "device", 14, norm_every=0, init=init, **_v5(T))
+
+
+@pytest.mark.parametrize("T", [3, 4])
+def test_graph_eager_stepwise_chunked_agree(T):
+    kw = _v5(T)
+    a = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=True, **kw)
+    b = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=False, **kw)
+    c = solve_gpu(516, 64, 2, "ring", "device", 30, 1, stepwise=True, **kw)
+    d = solve_gpu(516, 64, 2, "ring", "device", 30, 7, chunks_of_run=[3, 11, 16], **kw)
+    e = solve_gpu(516, 64, 2, "ring", "device", 30, 7, chunks_of_run=[5, 5, 5, 15], use_graph=False, **kw)
+    for x in (b, c, d, e):
+        for s1, s2 in zip(a["final"], x["final"]):
+            assert np.array_equal(bits(s1), bits(s2))
+    for x in (b, d, e):
+        assert np.array_equal(a["norms"], x["norms"])
+    assert np.array_equal(a["norms"], c["norms"][[0, 7, 14, 21, 28]])
+    _, want, want_norms = _oracle(516, 64, "ring", 30, 7)
+    assert_slabs_equal_global(a["final"], want, 2, "ring")
+    assert np.allclose(a["norms"], want_norms, rtol=NORM_RTOL, atol=0)
+
+
+def test_switch_variants_and_modes_mid_run():
+    """Variant 5 (T = 4, 3) <-> variant 4 <-> variant 1 on one solver; then variant 5 in host and
+    partial mode (one-iteration launches of the ghost-lane layout + NCCL / Acknowledge)."""
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+    from vranks import run_ranks
+    nx, ny, P = 1028, 64, 2
+
+    def body(rank, P, ag):
+        env = U.Env(rank, P, 0, ag)
+        comm = U.Comm(env, *U.ring_neighbours(rank, P))
+        st = torch.cuda.Stream()
+        coord = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
+        coord.set_timeout(5.0)
+        J = U.Jacobi(comm, nx, ny)
+        out = []
+        for v, T, it in ((5, 4, 10), (4, 0, 5), (5, 3, 7), (1, 0, 3), (5, 4, 9)):
+            J.set_launch(v, 0, 0, 0, T)
+            out.append(J.run(coord, it, 5))
+            coord.sync()
+        slab = J.copy_out(coord)
+        comm.barrier()
+        J.destroy()
+        coord.destroy()
+        comm.destroy()
+        env.finalize()
+        return slab, np.concatenate(out)
+
+    res = run_ranks(P, body)
+    _, want, want_norms = _oracle(nx, ny, "ring", 34, 5)
+    assert_slabs_equal_global([r[0] for r in res], want, P, "ring")
+    assert np.allclose(res[0][1], want_norms, rtol=NORM_RTOL, atol=0)
+
+    env = U.Env(0, 1, 0)
+    comm = U.Comm(env, 0, 0)
+    st = torch.cuda.Stream()
+    coords = {m: U.Coord(comm, v, st.cuda_stream) for m, v in (("device", 1), ("host", 0), ("partial", 2))}
+    J = U.Jacobi(comm, nx, ny)
+    J.set_launch(5, 0, 0, 0, 4)
+    for m, it in (("device", 8), ("host", 5), ("device", 6), ("partial", 3), ("device", 7), ("host", 2)):
+        J.run(coords[m], it, 0)
+        coords[m].sync()
+    out = J.copy_out(coords["device"])
+    J.destroy()
+    for c in coords.values():
+        c.destroy()
+    comm.destroy()
+    env.finalize()
+    _, want, _ = _oracle(nx, ny, "ring", 31, 0)
+    assert_slabs_equal_global([out], want, 1, "ring")
+
+
+@pytest.mark.parametrize("mode", ["host", "partial"])
+def test_host_and_partial_modes(mode):
+    _check(1028, 40, 1, "ring", mode, 11, norm_every=3, **_v5(4))
+
+
+def test_subnormal_front_no_ftz():
+    nx, ny = 96, 8
+    a = np.zeros((ny + 2, nx), np.float32)
+    a[:, 0] = 1.0
+    for k in (64, 70, 74, 75):
+        res = solve_gpu(nx, ny, 1, "ring", "device", k, 0, init=a, **_v5(4))
+        s = res["final"][0]
+        want = np.float32(2.0 ** (-2 * k)) if k <= 74 else np.float32(0.0)
+        assert s[1, k] == want and s[1, k + 1] == 0.0
+
+
+@pytest.mark.parametrize("T", [2, 3, 4])
+def test_full_size_16384(T):
+    """16384^2 (configs[2]/[3] at P = 1): whole grid bit-exact, norms on every level."""
+    _check(16384, 16384, 1, "ring", "device", 2 * T + 1, norm_every=T, **_v5(T))
+
+
+def test_config2_strong_16384_over_8_ranks():
+    _check(16384, 16384, 8, "ring", "device", 9, norm_every=4, **_v5(4))
+
+
+def test_config1_4096_2ranks_1000_iterations():
+    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, **_v5(4))
