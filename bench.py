@@ -60,7 +60,7 @@ def parse():
     ap.add_argument("--cpu-sample-iters", type=int, default=3)
     ap.add_argument("--variant", type=int, default=-1,
                     help="0 register march, 1 TMA-staged, 2 dynamic tiles, 3 persistent, 4 two iterations per "
-                         "launch (-1: library default = 4)")
+                         "launch, 5 T iterations per launch (T = --tile-rows; -1: library default = 5, T = 4)")
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--block-x", type=int, default=0)
@@ -227,10 +227,18 @@ def run_ours(a):
     ms_per_step = t_max / a.steps
     total_pts = pts_rank * world * ips * a.steps
     glups = total_pts / (t_max / 1e3) / 1e9
-    # two-iteration launches (variant 4, device mode, n >= 2, norm_every != 1) + an odd remainder
-    two = launch_info["variant"] == 4 and a.mode == "device" and n >= 2 and a.norm_every != 1
-    per_launch = 2 if two else 1
-    launches_per_step = ips // 2 + ips % 2 if two else ips
+    # iterations per launch: variant 4 = 2, variant 5 = T (device mode, n >= 2T, norm_every 0 or
+    # >= T), else 1; the last launch of a step may be shorter
+    v = launch_info["variant"]
+    per_launch = 1
+    if a.mode == "device" and v == 4 and n >= 2 and a.norm_every != 1:
+        per_launch = 2
+    elif a.mode == "device" and v == 5:
+        per_launch = launch_info["tile_rows"]
+        while per_launch > 1 and not (n >= 2 * per_launch and (a.norm_every <= 0 or a.norm_every >= per_launch)):
+            per_launch -= 1
+    two = per_launch > 1
+    launches_per_step = -(-ips // per_launch)
     launches = a.steps * launches_per_step + (
         a.steps * ((ips + a.norm_every - 1) // a.norm_every) if a.mode == "host" else 0)
 
@@ -240,8 +248,9 @@ def run_ours(a):
         buf = np.zeros(2, np.float64)
         for s, e in es:
             s.record(stream)
-            if iters_per_launch == 2:  # one two-iteration launch (norm_every 2: one norm round in it)
-                J.run(coord, 2, 2 if compute_norm else 0, False, norms_out=buf if compute_norm else None)
+            if iters_per_launch > 1:  # one multi-iteration launch (norm_every = T: one norm round in it)
+                J.run(coord, iters_per_launch, iters_per_launch if compute_norm else 0, False,
+                      norms_out=buf if compute_norm else None)
             else:
                 J.step(coord, compute_norm, buf if compute_norm else None)
             e.record(stream)
@@ -260,7 +269,8 @@ def run_ours(a):
     # last iterate written once -- 8 B per point per launch, for 1 or 2 iterations
     alg_bytes = 8.0 * pts_rank
     achieved = alg_bytes / (k_plain / 1e3) / 1e9
-    kname = "jacobi_two_step_kernel" if two else "jacobi_iter_kernel"
+    kname = {4: "jacobi_two_step_kernel", 5: f"jacobi_t_kernel<{per_launch}>"}.get(v, "jacobi_iter_kernel") if two \
+        else ("jacobi_t_kernel<1>" if v == 5 else "jacobi_iter_kernel")
     roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
             "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": ncu_traffic(nx, n, kname),
             "alg_bytes_per_launch": alg_bytes, "iterations_per_launch": per_launch,
@@ -270,7 +280,8 @@ def run_ours(a):
     if two:
         # the one-iteration kernel in the same geometry, for comparison (8 B per point per iteration)
         k1 = allreduce_max(dist, kernel_ms(False, 30, 1))
-        roof["one_iteration_kernel"] = {"kernel": "jacobi_iter_kernel", "kernel_ms": round(k1, 5),
+        roof["one_iteration_kernel"] = {"kernel": "jacobi_t_kernel<1>" if v == 5 else "jacobi_iter_kernel",
+                                        "kernel_ms": round(k1, 5),
                                         "achieved": round(alg_bytes / (k1 / 1e3) / 1e9, 1),
                                         "glups": round(pts_rank * world / (k1 / 1e3) / 1e9, 1)}
 
@@ -349,12 +360,12 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
     st = torch.cuda.Stream()
     co1 = U.Coord(comm1, mode, st.cuda_stream)
     J1 = U.Jacobi(comm1, nx, n)
-    J1.set_launch(launch_info["variant"], 0, 0, launch_info["stages"])
+    J1.set_launch(launch_info["variant"], 0, 0, launch_info["stages"], launch_info["tile_rows"])
     es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(30)]
     for s, e in es:
         s.record(st)
-        if per_launch == 2:
-            J1.run(co1, 2, 0, False)
+        if per_launch > 1:
+            J1.run(co1, per_launch, 0, False)
         else:
             J1.step(co1, False, None)
         e.record(st)

@@ -58,9 +58,19 @@ constexpr int kPad = UC_STAGE_PAD;  // staged ring: halo floats copied on each s
 #define UC_TWO_STEP_UNROLL 2
 #endif
 constexpr int kTwoStepUnroll = UC_TWO_STEP_UNROLL;
+// T-level kernel (variant 5): min blocks per SM (2: 113-register cap, no spills at T = 4) and
+// the unroll of the row loop (3 = the period of the register rotation: no moves); sweep in
+// profiles/r1_multi_step_sweep.txt
 #ifndef UC_T_MINBLOCKS
-#define UC_T_MINBLOCKS 3
+#define UC_T_MINBLOCKS 2
 #endif
+#ifndef UC_T_UNROLL
+#define UC_T_UNROLL 3
+#endif
+#ifndef UC_PACKED_F32X2
+#define UC_PACKED_F32X2 1
+#endif
+constexpr int kTUnroll = UC_T_UNROLL;
 #ifndef UC_TWO_STEP_MINBLOCKS
 #define UC_TWO_STEP_MINBLOCKS 3
 #endif
@@ -1036,14 +1046,46 @@ int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStrea
 
 constexpr int kOwned = 30;  // owned lanes per warp (lanes 1..30)
 
+// Packed fp32x2 arithmetic of sm_100 (FADD2 / FMUL2): two IEEE round-to-nearest operations per
+// instruction, no FTZ (no .ftz), never contracted -- bit-identical to two __fadd_rn / __fmul_rn.
+__device__ __forceinline__ void add2_rn(float a0, float a1, float b0, float b1, float& r0, float& r1) {
+  asm("{\n .reg .b64 a, b, r;\n mov.b64 a, {%2, %3};\n mov.b64 b, {%4, %5};\n"
+      " add.rn.f32x2 r, a, b;\n mov.b64 {%0, %1}, r;\n}"
+      : "=f"(r0), "=f"(r1) : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
+}
+__device__ __forceinline__ void quarter2_rn(float a0, float a1, float& r0, float& r1) {
+  asm("{\n .reg .b64 a, q, r;\n mov.b64 a, {%2, %3};\n mov.b64 q, {%4, %4};\n"
+      " mul.rn.f32x2 r, a, q;\n mov.b64 {%0, %1}, r;\n}"
+      : "=f"(r0), "=f"(r1) : "f"(a0), "f"(a1), "f"(0.25f));
+}
+
+// row_update for the ghost-lane layout (no cross-warp operand): new = 0.25f*((l+r)+(t+b)) with
+// the vertical sums t+b, the outer sums and the products packed two columns per instruction.
 __device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, int x4, int nx4) {
   const float L = __shfl_up_sync(kFull, c.w, 1);    // lane 0: its own value (ghost lane, discarded)
   const float R = __shfl_down_sync(kFull, c.x, 1);  // lane 31: likewise
+#if UC_PACKED_F32X2
+  const float hx = __fadd_rn(L, c.y), hy = __fadd_rn(c.x, c.z);
+  const float hz = __fadd_rn(c.y, c.w), hw = __fadd_rn(c.z, R);
+  float vx, vy, vz, vw, sx, sy, sz, sw, ox, oy, oz, ow;
+  add2_rn(up.x, up.y, dn.x, dn.y, vx, vy);
+  add2_rn(up.z, up.w, dn.z, dn.w, vz, vw);
+  add2_rn(hx, hy, vx, vy, sx, sy);
+  add2_rn(hz, hw, vz, vw, sz, sw);
+  quarter2_rn(sx, sy, ox, oy);
+  quarter2_rn(sz, sw, oz, ow);
+  float4 o;
+  o.x = (x4 == 0) ? c.x : ox;
+  o.y = oy;
+  o.z = oz;
+  o.w = (x4 == nx4 - 1) ? c.w : ow;
+#else
   float4 o;
   o.x = (x4 == 0) ? c.x : upd(L, c.y, up.x, dn.x);
   o.y = upd(c.x, c.z, up.y, dn.y);
   o.z = upd(c.y, c.w, up.z, dn.z);
   o.w = (x4 == nx4 - 1) ? c.w : upd(c.z, R, up.w, dn.w);
+#endif
   return o;
 }
 
@@ -1203,12 +1245,12 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
   RingCursor cur{0, 0u};
   float* out = dst + (size_t)a * pitch + 4 * (size_t)x4;  // the A_{k+T} row a comes out at i = 2T
   (void)lane;
-#pragma unroll 2
+#pragma unroll(kTUnroll)
   for (int i = 0; i < rows; ++i) {
     mbar_wait(full + cur.st, cur.ph);
     float4 nv = *reinterpret_cast<const float4*>(ring + (size_t)cur.st * ST + g.ring_off);
     __syncwarp();
-    if ((threadIdx.x & 31) == 0) mbar_arrive(empty + cur.st);
+    mbar_arrive_if(empty + cur.st, (threadIdx.x & 31) == 0);
     if (++cur.st == NS) {
       cur.st = 0;
       cur.ph ^= 1u;

@@ -88,13 +88,16 @@ struct JacobiParams {
 };
 
 constexpr int kFlagStride = 16;  // u64 per flag = 128 bytes, one flag per L2 line
-// Defaults from the round-1 sweeps at 16384^2 (profiles/r1_sweep.txt, r1_two_step_sweep.txt):
-// the TMA-staged march with a 3-row ring reaches 6.36 TB/s vs 6.07 for the register march
-// (deeper rings lose); the two-iteration kernel (variant 4, 3 blocks/SM, 4-row ring) moves the
-// same 8 B/point per launch at 6.4 TB/s for two iterations, so it is the default.
-constexpr int kDefaultVariant = 4;
+// Defaults from the round-1 sweeps at 16384^2 (profiles/r1_sweep.txt, r1_two_step_sweep.txt,
+// r1_multi_step_sweep.txt): the TMA-staged march with a 3-row ring reaches 6.36 TB/s vs 6.07 for
+// the register march (deeper rings lose); the two-iteration kernel (variant 4, 3 blocks/SM,
+// 4-row ring) moves the same 8 B/point per launch at 6.4 TB/s for two iterations; the T-level
+// ghost-lane kernel (variant 5, T = 4, 2 blocks/SM, 8-row ring) does four iterations per launch
+// at 0.40 ms, so it is the default.
+constexpr int kDefaultVariant = 5;
 constexpr int kDefaultStages = 3;
 constexpr int kDefaultStagesTwoStep = 4;
+constexpr int kDefaultStagesMulti = 8;
 constexpr int kDefaultTileRows = 64;
 
 // Launch wrappers implemented in kernels.cu

@@ -27,7 +27,7 @@ def window_oracle(nx, ny, y0, y1, k, topology="ring"):
     return out[k + 1:k + 1 + (y1 - y0 + 1)]
 
 
-@pytest.mark.parametrize("variant", [4, 1, 5])
+@pytest.mark.parametrize("variant", [5, 4, 1])
 def test_weak_scaling_8x16384sq_sampled_rows(variant):
     import torch
 
@@ -43,11 +43,11 @@ def test_weak_scaling_8x16384sq_sampled_rows(variant):
         co = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
         co.set_timeout(30.0)
         J = U.Jacobi(comm, nx, ny)
-        if variant != 4:
-            J.set_launch(variant)  # variant 5: T = 4 iterations per launch (k = 4: one launch)
+        if variant != 5:
+            J.set_launch(variant)
         try:
             comm.barrier()
-            J.run(co, k, 2, use_graph=True)
+            J.run(co, k, 4, use_graph=True)  # variant 5: one launch of T = 4 iterations
             co.sync()
             top = J.copy_rows(co, 0, edge + 1)                  # halo row 0 + owned rows 1..edge
             bot = J.copy_rows(co, n + 1 - edge, edge + 1)       # owned rows n-edge+1..n + halo n+1

@@ -266,12 +266,12 @@ def test_constant_field_fixed_and_zero_norm():
 # --------------------------------------------------------------------------- full size
 def test_full_size_16384_single_gpu_bench_configuration():
     """BASELINE.json configs[2]/[3] at P = 1 (16384^2 fp32, 1 GiB per slab), in the launch
-    configuration bench.py times (device mode, ring, CUDA graph, default geometry = variant 4,
-    two iterations per launch): the whole grid bit-exact vs the oracle after 6 and 7 iterations
-    (odd: a one-iteration launch at the end), norms within 1e-5 on both levels."""
-    res = _check(16384, 16384, 1, "ring", "device", 6, norm_every=3)
-    assert res["launch"]["variant"] == 4 and res["launch"]["stages"] == 4
-    _check(16384, 16384, 1, "ring", "device", 7, norm_every=2)
+    configuration bench.py times (device mode, ring, CUDA graph, default geometry = variant 5,
+    four iterations per launch, 8-row ring): the whole grid bit-exact vs the oracle after 8 and 11
+    iterations (a three-iteration launch at the end), norms within 1e-5 on every level."""
+    res = _check(16384, 16384, 1, "ring", "device", 8, norm_every=4)
+    assert res["launch"]["variant"] == 5 and res["launch"]["stages"] == 8 and res["launch"]["tile_rows"] == 4
+    _check(16384, 16384, 1, "ring", "device", 11, norm_every=5)
 
 
 def test_full_size_host_mode():
