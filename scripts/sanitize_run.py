@@ -26,14 +26,19 @@ def main():
         dict(P=1, mode="device", variant=1), dict(P=1, mode="device", variant=0), dict(P=1, mode="device", variant=2),
         dict(P=1, mode="device", variant=3), dict(P=1, mode="host", variant=1), dict(P=1, mode="partial", variant=1),
         dict(P=2, mode="device", variant=1), dict(P=2, mode="device", variant=3),
+        dict(P=1, mode="device", variant=4), dict(P=2, mode="device", variant=4),
+        dict(P=1, mode="device", variant=5, T=4, ne=4), dict(P=2, mode="device", variant=5, T=4, ne=4),
+        dict(P=2, mode="device", variant=5, T=3, ne=3), dict(P=1, mode="device", variant=5, T=2, ne=2),
+        dict(P=1, mode="host", variant=5, T=4), dict(P=1, mode="partial", variant=5, T=4),
     ]
     if len(sys.argv) > 1:
         cases = cases[: int(sys.argv[1])]
-    nx, ny, iters, ne = 132, 24, 4, 2
+    nx, ny, iters = 132, 24, 9
     for c in cases:
         P = c["P"]
+        ne = c.get("ne", 2)
         res = solve_gpu(nx, ny * P, P, "ring", c["mode"], iters, ne if c["mode"] != "partial" or P == 1 else 0,
-                        variant=c["variant"], use_graph=False)
+                        variant=c["variant"], tile_rows=c.get("T", 0), use_graph=False)
         want, _ = oracle.jacobi_run(gen.global_field(nx, ny * P, "ring"), iters, "ring")
         assert_slabs_equal_global(res["final"], want, P, "ring")
         print("ok", c, flush=True)
