@@ -9,13 +9,15 @@ Workload (BASELINE.json configs[3], weak scaling): 16384 x 16384 fp32 points per
 (rank r owns rows r*16384..), device-initiated halo exchange fused into the stencil, the global
 L2 norm every 100 iterations.  At N = 1 this is also configs[2]'s single-GPU point.
 A "step" = one pass of the whole hot path: 100 Jacobi iterations (stencil + halo exchange on
-every iteration, the norm allreduce on the first), launched as one cached CUDA graph.
+every iteration, the norm allreduce on the first), launched as one cached CUDA graph of 25
+launches of the default kernel (variant 5: four iterations per launch, every iteration's boundary
+rows exchanged; --variant 1 = one iteration per launch, the paper's structure).
 GLUPS = NY * (NX - 2) * 100 * K / t / 1e9 over all ranks; t = max over ranks of the CUDA-event
 time of the K timed steps (inputs > L2: 2 GiB working set per GPU vs 126 MB L2, no flush needed).
 
 Timing protocol: barrier + synchronize on both sides of the timed region, W >= 3 warm-up steps.
-Extra objects on the JSON line: roofline (dominant kernel = jacobi_iter_kernel, per-launch CUDA
-events), cpu_baseline (the oracle on this host, rank 0, N = 1), e2e (host-buffer end-to-end through
+Extra objects on the JSON line: roofline (dominant kernel = jacobi_t_kernel<4>, per-launch CUDA
+events, algorithmic bytes = 8 B per point per launch), cpu_baseline (the oracle on this host, rank 0, N = 1), e2e (host-buffer end-to-end through
 the C-ABI), clocks (nvidia-smi during the timed region), halo (exchange overlap).
 """
 from __future__ import annotations
@@ -127,7 +129,8 @@ class ClockSampler:
     def __init__(self, index: int):
         self.index = index
         self.proc = None
-        self.lines = []
+        self.lines = []   # (arrival time, line)
+        self.t0 = self.t1 = None
 
     def start(self):
         try:
@@ -141,7 +144,15 @@ class ClockSampler:
 
     def _read(self):
         for line in self.proc.stdout:
-            self.lines.append(line.strip())
+            self.lines.append((time.time(), line.strip()))
+
+    def mark_start(self):
+        """Started before the warm-up (nvidia-smi needs ~0.1-0.3 s to start); the timed region is
+        [mark_start, mark_stop] and only samples that arrive inside it count."""
+        self.t0 = time.time()
+
+    def mark_stop(self):
+        self.t1 = time.time()
 
     def stop(self):
         if self.proc is None:
@@ -153,7 +164,12 @@ class ClockSampler:
             self.proc.kill()
         sms, maxs, reasons, power = [], [], set(), []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for l in self.lines:
+        lines = self.lines
+        if self.t0 is not None and self.t1 is not None:
+            lines = [l for t, l in self.lines if self.t0 <= t <= self.t1 + 0.025]
+        else:
+            lines = [l for _, l in self.lines]
+        for l in lines:
             f = [x.strip() for x in l.split(",")]
             if len(f) < 9:
                 continue
@@ -204,15 +220,16 @@ def run_ours(a):
     def step():
         J.run(coord, ips, a.norm_every, use_graph, norms_out=norms_buf)
 
+    clocks = ClockSampler(local)
+    clocks.start()  # sampling from the warm-up on; only samples inside the timed region count
     for _ in range(a.warmup):
         step()
     coord.sync()
 
     # ---------------- timed region: K steps, events on the coordinator's stream
-    clocks = ClockSampler(local)
     barrier(dist)
     torch.cuda.synchronize()
-    clocks.start()
+    clocks.mark_start()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     for _ in range(a.steps):
@@ -220,6 +237,7 @@ def run_ours(a):
     e1.record(stream)
     coord.sync()
     torch.cuda.synchronize()
+    clocks.mark_stop()
     barrier(dist)
     clk = clocks.stop()
     t_ms = e0.elapsed_time(e1)

@@ -1061,6 +1061,7 @@ __device__ __forceinline__ void quarter2_rn(float a0, float a1, float& r0, float
 
 // row_update for the ghost-lane layout (no cross-warp operand): new = 0.25f*((l+r)+(t+b)) with
 // the vertical sums t+b, the outer sums and the products packed two columns per instruction.
+template <bool DIRI = true>
 __device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, int x4, int nx4) {
   const float L = __shfl_up_sync(kFull, c.w, 1);    // lane 0: its own value (ghost lane, discarded)
   const float R = __shfl_down_sync(kFull, c.x, 1);  // lane 31: likewise
@@ -1075,10 +1076,10 @@ __device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, i
   quarter2_rn(sx, sy, ox, oy);
   quarter2_rn(sz, sw, oz, ow);
   float4 o;
-  o.x = (x4 == 0) ? c.x : ox;
+  o.x = (DIRI && x4 == 0) ? c.x : ox;  // DIRI = false: no lane of the block holds a fixed column
   o.y = oy;
   o.z = oz;
-  o.w = (x4 == nx4 - 1) ? c.w : ow;
+  o.w = (DIRI && x4 == nx4 - 1) ? c.w : ow;
 #else
   float4 o;
   o.x = (x4 == 0) ? c.x : upd(L, c.y, up.x, dn.x);
@@ -1201,7 +1202,38 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
 
 // The T-level staged march: A_{k+T} rows a..b of strip s (rows outside the boundary rounds').
 // The producer streams the A_k rows a-T..b+T; consumers keep two rows per level.
-template <int T, int NL>
+// One row of the T-level march: take the next A_k row from the ring, advance every level, store
+// the A_{k+T} row (STORE: from the 2T-th row on).
+template <int T, int NL, bool DIRI, bool STORE>
+__device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
+                                       const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
+                                       float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+  mbar_wait(full + cur.st, cur.ph);
+  float4 nv = *reinterpret_cast<const float4*>(ring + (size_t)cur.st * ST + g.ring_off);
+  __syncwarp();
+  mbar_arrive_if(empty + cur.st, (threadIdx.x & 31) == 0);
+  if (++cur.st == NS) {
+    cur.st = 0;
+    cur.ph ^= 1u;
+  }
+#pragma unroll
+  for (int j = 0; j < T; ++j) {
+    const float4 o = row_update_g<DIRI>(w0[j], w1[j], nv, g.x4, nx4);  // level j+1, row r-j-1
+    if (NL == j + 1 && g.own) {
+      const int y = a - T + i - j - 1;
+      if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
+    }
+    w0[j] = w1[j];
+    w1[j] = nv;
+    nv = o;
+  }
+  if (STORE) {
+    if (g.own) st4(out, nv);
+    out += pitch;
+  }
+}
+
+template <int T, int NL, bool DIRI>
 __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src, float* dst, int s,
                                         const GhostLayout& g, int a, int b, double& acc, float* ring,
                                         uint64_t* full, uint64_t* empty, bool proxy_fence) {
@@ -1237,40 +1269,19 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
     }
     return;
   }
-  const int lane = threadIdx.x & 31;
-  const int x4 = g.x4, nx4 = p.nx4;
+  const int nx4 = p.nx4;
   float4 w0[T], w1[T];  // level j: rows r-j-1 (w0) and r-j (w1) before row r arrives
 #pragma unroll
   for (int j = 0; j < T; ++j) w0[j] = w1[j] = make_float4(0.f, 0.f, 0.f, 0.f);
   RingCursor cur{0, 0u};
-  float* out = dst + (size_t)a * pitch + 4 * (size_t)x4;  // the A_{k+T} row a comes out at i = 2T
-  (void)lane;
-#pragma unroll(kTUnroll)
-  for (int i = 0; i < rows; ++i) {
-    mbar_wait(full + cur.st, cur.ph);
-    float4 nv = *reinterpret_cast<const float4*>(ring + (size_t)cur.st * ST + g.ring_off);
-    __syncwarp();
-    mbar_arrive_if(empty + cur.st, (threadIdx.x & 31) == 0);
-    if (++cur.st == NS) {
-      cur.st = 0;
-      cur.ph ^= 1u;
-    }
+  float* out = dst + (size_t)a * pitch + 4 * (size_t)g.x4;  // the A_{k+T} row a comes out at i = 2T
+  // the first 2T rows only fill the levels (rows >= 2T + 1 since a <= b)
 #pragma unroll
-    for (int j = 0; j < T; ++j) {
-      const float4 o = row_update_g(w0[j], w1[j], nv, x4, nx4);  // level j+1, row r-j-1
-      if (NL == j + 1 && g.own) {
-        const int y = a - T + i - j - 1;
-        if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
-      }
-      w0[j] = w1[j];
-      w1[j] = nv;
-      nv = o;
-    }
-    if (i >= 2 * T) {
-      if (g.own) st4(out, nv);
-      out += pitch;
-    }
-  }
+  for (int i = 0; i < 2 * T; ++i)
+    t_step<T, NL, DIRI, false>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc);
+#pragma unroll(kTUnroll)
+  for (int i = 2 * T; i < rows; ++i)
+    t_step<T, NL, DIRI, true>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc);
 }
 
 template <int T, int NL>
@@ -1291,7 +1302,13 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
   if (bot_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, false, true, acc);
   const int a = max(lo, PT + 1);
   const int b = min(hi, p.n - PT);
-  if (a <= b) march_t<T, NL>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
+  if (a <= b) {
+    // fixed columns (0, NX-1) among the block's lanes, ghosts included: keep them fixed
+    const int xs4 = s * p.strip4;
+    const bool diri = xs4 <= 1 || xs4 + p.strip4 >= p.nx4 - 1;
+    if (diri) march_t<T, NL, true>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
+    else march_t<T, NL, false>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
+  }
   if ((top_blk || bot_blk) && (int)threadIdx.x < p.consumers) {
     for (int j = 2; j <= T; ++j) {  // consumers only (named barrier 1)
       if (top_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
