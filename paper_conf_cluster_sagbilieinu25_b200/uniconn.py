@@ -127,6 +127,16 @@ def chain_neighbours(rank: int, size: int):
     return (rank - 1 if rank > 0 else -1), (rank + 1 if rank < size - 1 else -1)
 
 
+def launch_plan(variant: int, levels: int, mode: int, n_local: int, iters: int, norm_every: int) -> list:
+    """uc_jacobi_launch_plan: iterations per launch of a uc_jacobi_run (host logic, no device)."""
+    cnt = lib.uc_jacobi_launch_plan(variant, levels, mode, n_local, iters, norm_every, None, 0)
+    if cnt < 0:
+        check(-cnt, "uc_jacobi_launch_plan")
+    buf = (C.c_int * max(1, cnt))()
+    lib.uc_jacobi_launch_plan(variant, levels, mode, n_local, iters, norm_every, buf, cnt)
+    return list(buf[:cnt])
+
+
 class SymMem:
     """Symmetric memory: same-size, peer-addressable on every rank."""
 
