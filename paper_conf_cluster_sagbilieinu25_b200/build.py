@@ -64,19 +64,31 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     nd = nccl_dir()
     os.makedirs(os.path.dirname(os.path.abspath(target)), exist_ok=True)
     tmp = target + f".tmp{os.getpid()}"
-    cmd = [nvcc(), *ARCH, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-shared", "-I", INCLUDE, "-I", CSRC,
-           "-I", os.path.join(nd, "include"),
-           *sources(), "-o", tmp, "-L", os.path.join(nd, "lib"), "-l:libnccl.so.2",
-           "-Xlinker", "-rpath=" + os.path.join(nd, "lib")]
-    res = subprocess.run(cmd, capture_output=True, text=True)
+    objdir = os.path.join(ROOT, "build", "obj", os.path.basename(target) + f".{os.getpid()}")
+    os.makedirs(objdir, exist_ok=True)
+    flags = [*ARCH, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", INCLUDE, "-I", CSRC,
+             "-I", os.path.join(nd, "include")]
+    # one nvcc per translation unit, in parallel (the kernel TUs dominate the build time)
+    jobs = [(src, os.path.join(objdir, os.path.basename(src) + ".o")) for src in sources()]
+    cmds = [[nvcc(), *flags, "-c", src, "-o", obj] for src, obj in jobs]
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=max(1, min(len(cmds), os.cpu_count() or 1))) as ex:
+        results = list(ex.map(lambda c: subprocess.run(c, capture_output=True, text=True), cmds))
+    link = [nvcc(), *ARCH, "-shared", *[o for _, o in jobs], "-o", tmp, "-L", os.path.join(nd, "lib"),
+            "-l:libnccl.so.2", "-Xlinker", "-rpath=" + os.path.join(nd, "lib")]
+    if all(r.returncode == 0 for r in results):
+        results.append(subprocess.run(link, capture_output=True, text=True))
+        cmds.append(link)
     log = os.path.join(CSRC, "build.log")
     with open(log, "w") as f:
-        f.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
-    if res.returncode != 0:
-        sys.stderr.write(res.stdout + res.stderr)
+        for c, r in zip(cmds, results):
+            f.write(" ".join(c) + "\n" + r.stdout + r.stderr)
+    shutil.rmtree(objdir, ignore_errors=True)
+    if any(r.returncode != 0 for r in results):
+        sys.stderr.write("".join(r.stdout + r.stderr for r in results if r.returncode != 0))
         raise RuntimeError(f"nvcc failed (see {log})")
     if verbose:
-        sys.stderr.write(res.stderr)
+        sys.stderr.write("".join(r.stderr for r in results))
     os.replace(tmp, target)
     if out is None:
         build_examples()

@@ -104,6 +104,8 @@ constexpr int kDefaultTileRows = 64;
 int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_t(const JacobiParams& p, int grid, int block, int T, cudaStream_t s);
+int preload_multistep();                                             // multistep.cu
+int multistep_occupancy(int block, size_t smem, int* blocks_per_sm); // the deepest instance bounds all T
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
