@@ -9,15 +9,17 @@ Workload (BASELINE.json configs[3], weak scaling): 16384 x 16384 fp32 points per
 (rank r owns rows r*16384..), device-initiated halo exchange fused into the stencil, the global
 L2 norm every 100 iterations.  At N = 1 this is also configs[2]'s single-GPU point.
 A "step" = one pass of the whole hot path: 100 Jacobi iterations (stencil + halo exchange on
-every iteration, the norm allreduce on the first), launched as one cached CUDA graph of 25
-launches of the default kernel (variant 5: four iterations per launch, every iteration's boundary
-rows exchanged; --variant 1 = one iteration per launch, the paper's structure).
+every iteration, the norm allreduce on the first), launched as one cached CUDA graph of 17
+launches of the default kernel (variant 5: six iterations per launch -- 16 x 6 + 4 -- every
+iteration's boundary rows exchanged; --tile-rows T picks T = 1..8 iterations per launch;
+--variant 1 = one iteration per launch, the paper's structure).
 GLUPS = NY * (NX - 2) * 100 * K / t / 1e9 over all ranks; t = max over ranks of the CUDA-event
 time of the K timed steps (inputs > L2: 2 GiB working set per GPU vs 126 MB L2, no flush needed).
 
 Timing protocol: barrier + synchronize on both sides of the timed region, W >= 3 warm-up steps.
-Extra objects on the JSON line: roofline (dominant kernel = jacobi_t_kernel<4>, per-launch CUDA
-events, algorithmic bytes = 8 B per point per launch), cpu_baseline (the oracle on this host, rank 0, N = 1), e2e (host-buffer end-to-end through
+Extra objects on the JSON line: roofline (dominant kernel = jacobi_t_kernel<6, 2>, per-launch CUDA
+events, algorithmic bytes = 8 B per point per launch; roofline.alu = the same launch against the
+FP32-pipe peak), cpu_baseline (the oracle on this host, rank 0, N = 1), e2e (host-buffer end-to-end through
 the C-ABI), clocks (nvidia-smi during the timed region), halo (exchange overlap).
 """
 from __future__ import annotations
@@ -59,6 +61,7 @@ def parse():
                     help="TEST ONLY: put every rank on cuda:0 (exercises the multi-process path on a 1-GPU box; "
                          "ranks time-slice the GPU, so the numbers are not a benchmark)")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
+    ap.add_argument("--halo-only", action="store_true", help="skip e2e / cpu_baseline, keep the halo leg")
     ap.add_argument("--cpu-sample-iters", type=int, default=3)
     ap.add_argument("--variant", type=int, default=-1,
                     help="0 register march, 1 TMA-staged, 2 dynamic tiles, 3 persistent, 4 two iterations per "
@@ -106,6 +109,16 @@ def measured_peaks():
             d = json.load(f)
         return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy)"
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def sm_max_mhz():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        if d.get("sm_max_mhz"):
+            return float(d["sm_max_mhz"])
+    return 1965.0  # B200 max SM clock (B200_PROFILING.md)
 
 
 def ncu_traffic(nx, n, kernel="jacobi_iter_kernel"):
@@ -287,18 +300,30 @@ def run_ours(a):
     # last iterate written once -- 8 B per point per launch, for 1 or 2 iterations
     alg_bytes = 8.0 * pts_rank
     achieved = alg_bytes / (k_plain / 1e3) / 1e9
-    kname = {4: "jacobi_two_step_kernel", 5: f"jacobi_t_kernel<{per_launch}>"}.get(v, "jacobi_iter_kernel") if two \
-        else ("jacobi_t_kernel<1>" if v == 5 else "jacobi_iter_kernel")
+    # variant 5 ghost layout: G = 2 ghost lanes per warp side when T > 4 (28 of 32 lanes owned)
+    ghosts = 2 if v == 5 and launch_info["tile_rows"] > 4 else 1
+    kname = {4: "jacobi_two_step_kernel", 5: f"jacobi_t_kernel<{per_launch}, {ghosts}>"}.get(v, "jacobi_iter_kernel") \
+        if two else (f"jacobi_t_kernel<1, {ghosts}>" if v == 5 else "jacobi_iter_kernel")
     roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
             "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": ncu_traffic(nx, n, kname),
             "alg_bytes_per_launch": alg_bytes, "iterations_per_launch": per_launch,
             "hbm_bytes_per_point_iteration": 8.0 / per_launch,
             "kernel_ms": round(k_plain, 5), "kernel_norm_ms": round(k_norm, 5),
             "kernel_share_of_step": round(k_avg * launches_per_step / ms_per_step, 4), "peak_source": peak_src}
+    # the FP32-pipe roof beside it: 4 FP32 operations per point-iteration (3 FADD +
+    # 1 FMUL, never fused), T iterations per launch, ghost lanes compute too (x 32 / (32 - 2G));
+    # peak = SMs x 128 FP32 lanes x max SM clock
+    sms = torch.cuda.get_device_properties(local).multi_processor_count
+    alu_peak = sms * 128 * sm_max_mhz() * 1e6 / 1e12
+    ops = 4.0 * pts_rank * per_launch * (32.0 / (32 - 2 * ghosts) if v == 5 else 1.0)
+    alu = ops / (k_plain / 1e3) / 1e12
+    roof["alu"] = {"bound": "alu", "achieved": round(alu, 3), "peak": round(alu_peak, 2), "unit": "TFLOP/s",
+                   "frac": round(alu / alu_peak, 4), "flops_per_launch": ops,
+                   "peak_source": f"{sms} SMs x 128 FP32 lanes x {sm_max_mhz():.0f} MHz"}
     if two:
         # the one-iteration kernel in the same geometry, for comparison (8 B per point per iteration)
         k1 = allreduce_max(dist, kernel_ms(False, 30, 1))
-        roof["one_iteration_kernel"] = {"kernel": "jacobi_t_kernel<1>" if v == 5 else "jacobi_iter_kernel",
+        roof["one_iteration_kernel"] = {"kernel": f"jacobi_t_kernel<1, {ghosts}>" if v == 5 else "jacobi_iter_kernel",
                                         "kernel_ms": round(k1, 5),
                                         "achieved": round(alg_bytes / (k1 / 1e3) / 1e9, 1),
                                         "glups": round(pts_rank * world / (k1 / 1e3) / 1e9, 1)}
@@ -306,15 +331,21 @@ def run_ours(a):
     # ---------------- halo exchange overlap (differential, §8 d): same slab, no neighbours
     halo = None
     if not a.no_extras:
+        def full_launch():  # one launch of the timed configuration (T iterations, no norm)
+            if per_launch > 1:
+                J.run(coord, per_launch, 0, False)
+            else:
+                J.step(coord, False, None)
+
         halo = halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_plain, per_launch,
-                            launch_info)
+                            launch_info, full_launch, stream)
 
     # ---------------- e2e through the C-ABI with pinned host buffers
     # Every step: H2D of the step's input slab (pinned), the 100 iterations, D2H of the final slab
     # and the norms.  Two solvers on two streams alternate steps, so step i+1's H2D overlaps step
     # i's compute and D2H (both copy engines busy); the serial single-stream figure is kept too.
     e2e = None
-    if not a.no_extras:
+    if not a.no_extras and not a.halo_only:
         slab_elems = (n + 2) * nx
         ke = max(4, min(a.steps, 6))
         J2 = U.Jacobi(comm, nx, ny)
@@ -375,7 +406,7 @@ def run_ours(a):
 
     # ---------------- oracle on the host cores (rank 0, N = 1)
     cpu = None
-    if rank == 0 and world == 1 and not a.no_extras:
+    if rank == 0 and world == 1 and not a.no_extras and not a.halo_only:
         cpu = cpu_baseline(nx, a.ny_per_gpu, a.cpu_sample_iters)
 
     if rank == 0:
@@ -400,11 +431,14 @@ def run_ours(a):
         dist.destroy_process_group()
 
 
-def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full, per_launch, launch_info):
+def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full, per_launch, launch_info,
+                 full_launch=None, full_stream=None):
     """hidden = clamp(1 - (T_full - T_compute) / T_xchg, 0, 1) (SURVEY §8 d).  T_compute: the same
     slab and kernel with no neighbours (chain-less comm: top = bottom = -1 is not a valid Jacobi
     topology for P > 1, so we time a P = 1 dirichlet-chain solver of the same n rows in its own
-    communicator); T_xchg: the exchange alone = put_signal of one row to each neighbour."""
+    communicator); T_xchg: the exchange alone = put_signal of one row to each neighbour.
+    T_full and T_compute are timed in alternation (10 repetitions of 5 launches each, the
+    lowest and highest dropped, the mean of the rest), so clock drift cancels."""
     # T_compute: independent single-rank chain (no waits, no puts) on this GPU
     env1 = U.Env(0, 1, local)
     comm1 = U.Comm(env1, -1, -1)
@@ -412,21 +446,40 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
     co1 = U.Coord(comm1, mode, st.cuda_stream)
     J1 = U.Jacobi(comm1, nx, n)
     J1.set_launch(launch_info["variant"], 0, 0, launch_info["stages"], launch_info["tile_rows"])
-    es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(30)]
-    for s, e in es:
-        s.record(st)
+
+    def comp_launch():
         if per_launch > 1:
             J1.run(co1, per_launch, 0, False)
         else:
             J1.step(co1, False, None)
-        e.record(st)
-    co1.sync()
-    t_comp = statistics.mean(s.elapsed_time(e) for s, e in es[5:])
+
+    def timed(fn, stream, k=5):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(k):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / k
+
+    def trimmed(xs):
+        xs = sorted(xs)[1:-1] if len(xs) > 2 else xs
+        return statistics.mean(xs)
+
+    for _ in range(3):
+        comp_launch()
+    fulls, comps = [], []
+    for _ in range(10):
+        if full_launch is not None:
+            barrier(dist)
+            fulls.append(timed(full_launch, full_stream))
+        comps.append(timed(comp_launch, st))
+    t_comp = trimmed(comps)
+    t_full = trimmed(fulls) if fulls else k_full
     J1.destroy()
     co1.destroy()
     comm1.destroy()
     env1.finalize()
-    t_full = k_full
     # T_xchg: two row puts + signal waits (device mode), the same message size
     comm = U.Comm(env, *U.ring_neighbours(rank, world))
     st2 = torch.cuda.Stream()

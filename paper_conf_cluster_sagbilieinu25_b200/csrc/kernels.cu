@@ -1265,8 +1265,8 @@ int jacobi_occupancy(int variant, int block, size_t smem, int* blocks_per_sm) {
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_persistent_kernel, block, smem));
   else if (variant == 4)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_two_step_kernel, block, smem));
-  else if (variant == 5)  // the deepest (largest) instance bounds the geometry of all T
-    return multistep_occupancy(block, smem, blocks_per_sm);
+  else if (variant == 5)  // the deepest (largest) instance of the one-ghost layout
+    return multistep_occupancy(block, smem, 1, blocks_per_sm);
   else if (variant == 2)
     UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_iter_kernel<2>, block, smem));
   else if (variant == 1)

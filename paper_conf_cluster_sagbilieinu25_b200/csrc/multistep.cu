@@ -1,387 +1,46 @@
-// multistep.cu -- kernel variant 5 of libuniconn_b200: T Jacobi iterations per launch.
-// (§VI-C stencil; Listing 3 P:52-74 halo exchange, once per iteration.)
-#include "stencil_common.cuh"
+// multistep.cu -- kernel variant 5 of libuniconn_b200, G = 1 ghost lane per warp side (T = 1..4
+// iterations per launch), and the host-side dispatch of both ghost layouts (multistep_g2.cu:
+// G = 2, T = 1..8).  (§VI-C stencil; Listing 3 P:52-74 halo exchange.)
+#include "multistep.cuh"
 
 namespace uc {
 
-// ------------------------------------------------------------------------------ T iterations per launch
-// Variant 5: one launch advances A_k -> A_{k+T}, T = 1..4 (temporal blocking of depth T).  The
-// staged march keeps T register levels: from the A_k row r streamed through the TMA ring it
-// computes the A_{k+1} row r-1, the A_{k+2} row r-2, ..., and stores only the A_{k+T} row r-T:
-// 8 HBM bytes per point per launch, 8/T per point-iteration.
-//
-// Horizontal neighbours across warp edges: "ghost lanes".  A warp owns the 30 float4 columns of
-// its lanes 1..30; lanes 0 and 31 hold copies of the neighbouring warps' (or strips') edge
-// columns, loaded from the ring, and run the same stencil.  Their own results go wrong one column
-// per level from the outer side (their missing neighbour), so after T <= 4 levels the 4 columns
-// of a ghost lane may be wrong but every owned lane is exact: no cross-warp exchange, no barrier.
-// A strip is 30 * (consumers / 32) float4 columns (the last warps of a block may own fewer).
-//
-// Boundary rows: level j (A_{k+j}) rows near the slab edge depend on the neighbour's level j-1
-// rows, so the first/last row-chunk block of each strip runs T "rounds" per side: round j waits
-// for the neighbour's level j-1 edge row (round 1: the A_k halo row), recomputes levels 1..j of
-// the first few rows from A_k and the neighbour's rows, and puts its own level j edge row to the
-// neighbour (levels < T: the h buffers; level T: the halo row of the output slab) with a
-// release flag k + j.  Round 1 runs before the march (its puts overlap the whole sweep), rounds
-// 2..T after it.  Every level of every boundary row is exchanged, as in the one-iteration
-// kernel: only the HBM traffic of the interior changes.
-
-constexpr int kOwned = 30;  // owned lanes per warp (lanes 1..30)
-
-// Packed fp32x2 arithmetic of sm_100 (FADD2 / FMUL2): two IEEE round-to-nearest operations per
-// instruction, no FTZ (no .ftz), never contracted -- bit-identical to two __fadd_rn / __fmul_rn.
-__device__ __forceinline__ void add2_rn(float a0, float a1, float b0, float b1, float& r0, float& r1) {
-  asm("{\n .reg .b64 a, b, r;\n mov.b64 a, {%2, %3};\n mov.b64 b, {%4, %5};\n"
-      " add.rn.f32x2 r, a, b;\n mov.b64 {%0, %1}, r;\n}"
-      : "=f"(r0), "=f"(r1) : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
-}
-__device__ __forceinline__ void quarter2_rn(float a0, float a1, float& r0, float& r1) {
-  asm("{\n .reg .b64 a, q, r;\n mov.b64 a, {%2, %3};\n mov.b64 q, {%4, %4};\n"
-      " mul.rn.f32x2 r, a, q;\n mov.b64 {%0, %1}, r;\n}"
-      : "=f"(r0), "=f"(r1) : "f"(a0), "f"(a1), "f"(0.25f));
-}
-
-// row_update for the ghost-lane layout (no cross-warp operand): new = 0.25f*((l+r)+(t+b)) with
-// the vertical sums t+b, the outer sums and the products packed two columns per instruction.
-template <bool DIRI = true>
-__device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, int x4, int nx4) {
-  const float L = __shfl_up_sync(kFull, c.w, 1);    // lane 0: its own value (ghost lane, discarded)
-  const float R = __shfl_down_sync(kFull, c.x, 1);  // lane 31: likewise
-#if UC_PACKED_F32X2
-  const float hx = __fadd_rn(L, c.y), hy = __fadd_rn(c.x, c.z);
-  const float hz = __fadd_rn(c.y, c.w), hw = __fadd_rn(c.z, R);
-  float vx, vy, vz, vw, sx, sy, sz, sw, ox, oy, oz, ow;
-  add2_rn(up.x, up.y, dn.x, dn.y, vx, vy);
-  add2_rn(up.z, up.w, dn.z, dn.w, vz, vw);
-  add2_rn(hx, hy, vx, vy, sx, sy);
-  add2_rn(hz, hw, vz, vw, sz, sw);
-  quarter2_rn(sx, sy, ox, oy);
-  quarter2_rn(sz, sw, oz, ow);
-  float4 o;
-  o.x = (DIRI && x4 == 0) ? c.x : ox;  // DIRI = false: no lane of the block holds a fixed column
-  o.y = oy;
-  o.z = oz;
-  o.w = (DIRI && x4 == nx4 - 1) ? c.w : ow;
-#else
-  float4 o;
-  o.x = (x4 == 0) ? c.x : upd(L, c.y, up.x, dn.x);
-  o.y = upd(c.x, c.z, up.y, dn.y);
-  o.z = upd(c.y, c.w, up.z, dn.z);
-  o.w = (x4 == nx4 - 1) ? c.w : upd(c.z, R, up.w, dn.w);
-#endif
-  return o;
-}
-
-struct GhostLayout {
-  int x4;        // float4 column of this thread (ghost lanes: the neighbour's edge column)
-  bool in_grid;  // 0 <= x4 < nx4 (may be loaded)
-  bool own;      // owned column of this strip: stored, put, counted in the norm
-  int ring_off;  // float offset of x4 in a ring row (ring row starts at column 4*xs4 - kPad)
-};
-__device__ __forceinline__ GhostLayout ghost_layout(const JacobiParams& p, int s) {
-  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-  const int xs4 = s * p.strip4;
-  const int xe4 = min(xs4 + p.strip4, p.nx4);
-  GhostLayout g;
-  g.x4 = xs4 + w * kOwned + lane - 1;
-  g.in_grid = g.x4 >= 0 && g.x4 < p.nx4;
-  g.own = lane >= 1 && lane <= kOwned && g.x4 < xe4 && t < p.consumers;
-  g.ring_off = 4 * (w * kOwned + lane);
-  return g;
-}
-
-// Row chunk q of the slab, first/last chunks shortened by p.chunk_shrink rows (their blocks
-// also run the boundary rounds).
-__device__ __forceinline__ void chunk_rows(const JacobiParams& p, int q, int& lo, int& hi) {
-  const long long nv = (long long)p.n + 2LL * p.chunk_shrink;
-  const long long a = (long long)q * nv / p.chunks - p.chunk_shrink;
-  const long long b = (long long)(q + 1) * nv / p.chunks - p.chunk_shrink;
-  lo = 1 + (int)max(0LL, min(a, (long long)p.n));
-  hi = (int)max(0LL, min(b, (long long)p.n));
-}
-
-// One boundary round j (1..T) of one side.  Rows are counted from the slab edge inward:
-// i = 0 is the halo row (top: slab row 0, bottom: slab row n+1), i = 1 the edge row (row 1 / n).
-// The stencil is symmetric in t and b, so the mirrored order gives bit-identical values.
-template <int T, int NL>
-__device__ __forceinline__ void t_round(const JacobiParams& p, const float* src, float* dst, int np, int s,
-                                        const GhostLayout& g, uint64_t k, int j, bool top, bool cta_sync,
-                                        double& acc) {
-  constexpr int PT = T > 1 ? T - 1 : 1;  // edge rows of A_{k+T} produced here (1..PT)
-  constexpr int NR = PT + T + 1;         // A_k rows 0..PT+T read
-  const bool has = top ? p.has_top : p.has_bot;
-  const bool dev = p.device_mode == 1;
-  const size_t pitch = (size_t)p.nx;
-  const int side = top ? 0 : 1;          // our h rows: 0 = from top, 1 = from bottom
-  if (threadIdx.x == 0 && has && dev) {
-    if (j == 1) wait_strip_flags(p, top ? 0 : p.flag_half, s, k);  // A_k halo rows
-    else {  // the neighbour's level j-1 edge row (its round j-1)
-      const uint64_t* f = p.h1_flags + (size_t)(j - 2) * 2 * p.flag_half * kFlagStride;
-      const int base = top ? 0 : p.flag_half;
-      const int s0 = s > 0 ? s - 1 : 0, s1 = s + 1 < p.strips ? s + 1 : s;
-      for (int q = s0; q <= s1; ++q) wait_ge(f + (size_t)(base + q) * kFlagStride, k + j - 1, p.timeout_ns, p.err);
-    }
-  }
-  if (cta_sync) __syncthreads();
-  else named_barrier_sync(1, p.consumers);
-  if ((int)threadIdx.x >= p.consumers) return;  // the producer warp (cta_sync rounds only)
-  float4 a[NR];
-#pragma unroll
-  for (int i = 0; i < NR; ++i) {
-    const int y = top ? i : p.n + 1 - i;
-    a[i] = g.in_grid ? reinterpret_cast<const float4*>(src + (size_t)y * pitch)[g.x4] : make_float4(0.f, 0.f, 0.f, 0.f);
-  }
-#pragma unroll
-  for (int m = 1; m <= T; ++m) {
-    if (m <= j) {
-      // level m rows 1 .. NR-1-m from level m-1 rows 0 .. NR-m (in place, ascending)
-      float4 prev = a[0];
-#pragma unroll
-      for (int i = 1; i < NR - m; ++i) {
-        const float4 o = row_update_g(prev, a[i], a[i + 1], g.x4, p.nx4);
-        if (NL == m && m == j && i <= PT && g.own) acc_sq(acc, o, a[i]);
-        prev = a[i];
-        a[i] = o;
-      }
-      // level m row 0: the neighbour's (waited for in round m+1 <= j), or the fixed row
-      if (m < j && has && g.in_grid)
-        a[0] = reinterpret_cast<const float4*>(p.h1_rows + ((size_t)(m - 1) * 2 + side) * pitch)[g.x4];
-    }
-  }
-  const bool put = has && p.device_mode != 0;
-  if (j < T) {
-    // our level j edge row -> the neighbour's h row of level j (top neighbour: its "from bottom")
-    if (put && g.own) {
-      float* nb = (top ? p.top_h1_rows : p.bot_h1_rows) + ((size_t)(j - 1) * 2 + (top ? 1 : 0)) * pitch;
-      reinterpret_cast<float4*>(nb)[g.x4] = a[1];
-    }
-  } else {
-#pragma unroll
-    for (int i = 1; i <= PT; ++i) {
-      const int y = top ? i : p.n + 1 - i;
-      if (g.own) reinterpret_cast<float4*>(dst + (size_t)y * pitch)[g.x4] = a[i];
-    }
-    if (put && g.own) {
-      if (top) reinterpret_cast<float4*>(p.top_slab[np] + (size_t)(p.n + 1) * pitch)[g.x4] = a[1];
-      else reinterpret_cast<float4*>(p.bot_slab[np])[g.x4] = a[1];
-    }
-  }
-  if (has && dev) {
-    named_barrier_sync(1, p.consumers);
-    if (threadIdx.x == 0) {
-      __threadfence_system();
-      if (j < T) {
-        uint64_t* f = (top ? p.top_h1_flags : p.bot_h1_flags) + (size_t)(j - 1) * 2 * p.flag_half * kFlagStride;
-        st_release_sys(f + (size_t)((top ? p.flag_half : 0) + s) * kFlagStride, k + j);
-      } else if (top) {
-        st_release_sys(p.top_flags + (size_t)(p.flag_half + s) * kFlagStride, k + T);  // top's from_bottom[s]
-      } else {
-        st_release_sys(p.bot_flags + (size_t)s * kFlagStride, k + T);                  // bottom's from_top[s]
-      }
-    }
-  }
-}
-
-// The T-level staged march: A_{k+T} rows a..b of strip s (rows outside the boundary rounds').
-// The producer streams the A_k rows a-T..b+T; consumers keep two rows per level.
-// One row of the T-level march: take the next A_k row from the ring, advance every level, store
-// the A_{k+T} row (STORE: from the 2T-th row on).
-template <int T, int NL, bool DIRI, bool STORE>
-__device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
-                                       const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
-                                       float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
-  mbar_wait(full + cur.st, cur.ph);
-  float4 nv = *reinterpret_cast<const float4*>(ring + (size_t)cur.st * ST + g.ring_off);
-  __syncwarp();
-  mbar_arrive_if(empty + cur.st, (threadIdx.x & 31) == 0);
-  if (++cur.st == NS) {
-    cur.st = 0;
-    cur.ph ^= 1u;
-  }
-#pragma unroll
-  for (int j = 0; j < T; ++j) {
-    const float4 o = row_update_g<DIRI>(w0[j], w1[j], nv, g.x4, nx4);  // level j+1, row r-j-1
-    if (NL == j + 1 && g.own) {
-      const int y = a - T + i - j - 1;
-      if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
-    }
-    w0[j] = w1[j];
-    w1[j] = nv;
-    nv = o;
-  }
-  if (STORE) {
-    if (g.own) st4(out, nv);
-    out += pitch;
-  }
-}
-
-template <int T, int NL, bool DIRI>
-__device__ __forceinline__ void march_t(const JacobiParams& p, const float* src, float* dst, int s,
-                                        const GhostLayout& g, int a, int b, double& acc, float* ring,
-                                        uint64_t* full, uint64_t* empty, bool proxy_fence) {
-  const int nc = p.consumers, NS = p.stages;
-  const int ST = 4 * nc + 2 * kPad;
-  const size_t pitch = (size_t)p.nx;
-  const int rows = b - a + 1 + 2 * T;
-  if ((int)threadIdx.x >= nc) {
-    if ((threadIdx.x & 31) == 0) {
-      const int xs = 4 * s * p.strip4;
-      const int xe = min(xs + 4 * p.strip4, p.nx);
-      const int left = xs >= kPad ? xs - kPad : 0;
-      const int right = min(xe + kPad, p.nx);
-      const unsigned bytes = (unsigned)(right - left) * 4u;
-      const int off = left - (xs - kPad);
-#if UC_L2_EVICT_FIRST
-      const uint64_t pol = policy_evict_first();
-#else
-      const uint64_t pol = policy_evict_normal();
-#endif
-      if (proxy_fence) fence_proxy_async_global();
-      int st = 0;
-      unsigned ph = 0;
-      for (int i = 0; i < rows; ++i) {
-        if (i >= NS) mbar_wait(empty + st, ph ^ 1u);
-        mbar_arrive_expect_tx(full + st, bytes);
-        bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(a - T + i) * pitch + left, bytes, full + st, pol);
-        if (++st == NS) {
-          st = 0;
-          ph ^= 1u;
-        }
-      }
-    }
-    return;
-  }
-  const int nx4 = p.nx4;
-  float4 w0[T], w1[T];  // level j: rows r-j-1 (w0) and r-j (w1) before row r arrives
-#pragma unroll
-  for (int j = 0; j < T; ++j) w0[j] = w1[j] = make_float4(0.f, 0.f, 0.f, 0.f);
-  RingCursor cur{0, 0u};
-  float* out = dst + (size_t)a * pitch + 4 * (size_t)g.x4;  // the A_{k+T} row a comes out at i = 2T
-  // the first 2T rows only fill the levels (rows >= 2T + 1 since a <= b)
-#pragma unroll
-  for (int i = 0; i < 2 * T; ++i)
-    t_step<T, NL, DIRI, false>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc);
-#pragma unroll(kTUnroll)
-  for (int i = 2 * T; i < rows; ++i)
-    t_step<T, NL, DIRI, true>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc);
-}
-
-template <int T, int NL>
-__device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int par, float* ring, uint64_t* full,
-                                         uint64_t* empty) {
-  constexpr int PT = T > 1 ? T - 1 : 1;
-  const float* src = p.slab[par];
-  float* dst = p.slab[par ^ 1];
-  const int s = blockIdx.x % p.strips;
-  const int q = blockIdx.x / p.strips;
-  const GhostLayout g = ghost_layout(p, s);
-  int lo, hi;
-  chunk_rows(p, q, lo, hi);
-  const bool top_blk = q == 0, bot_blk = q == p.chunks - 1;
-  double acc = 0.0;
-  // round 1 before the march (all threads: the producer must not read halo rows before the wait)
-  if (top_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, true, true, acc);
-  if (bot_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, false, true, acc);
-  const int a = max(lo, PT + 1);
-  const int b = min(hi, p.n - PT);
-  if (a <= b) {
-    // fixed columns (0, NX-1) among the block's lanes, ghosts included: keep them fixed
-    const int xs4 = s * p.strip4;
-    const bool diri = xs4 <= 1 || xs4 + p.strip4 >= p.nx4 - 1;
-    if (diri) march_t<T, NL, true>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
-    else march_t<T, NL, false>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
-  }
-  if ((top_blk || bot_blk) && (int)threadIdx.x < p.consumers) {
-    for (int j = 2; j <= T; ++j) {  // consumers only (named barrier 1)
-      if (top_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
-      if (bot_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, false, false, acc);
-    }
-  }
-  return acc;
-}
-
-// T iterations per launch.  Device mode: T = 1..4 (n >= 2T-1, at most one norm round per launch);
-// host / partial mode: T = 1 (the host API exchanges the halos after the kernel).
-template <int T>
-__global__ void __launch_bounds__(kMaxBlock + 32, UC_T_MINBLOCKS) jacobi_t_kernel(const JacobiParams p) {
-  __shared__ double smem[32];
-  __shared__ int s_last;
-  extern __shared__ __align__(128) unsigned char dyn[];
-  const int NS = p.stages;
-  uint64_t* full = reinterpret_cast<uint64_t*>(dyn);
-  uint64_t* empty = full + NS;
-  float* ring = reinterpret_cast<float*>(dyn + ((32 * NS + 127) / 128) * 128);
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < NS; ++i) {
-      mbar_init(full + i, 1);
-      mbar_init(empty + i, p.consumers / 32);
-    }
-    fence_mbar_init();
-  }
-  __syncthreads();
-  const uint64_t k = p.k_dev[0];
-  const int par = (int)((k + p.k_dev[2]) & 1);
-  int nl = 0;  // level (1..T) whose iteration k+nl-1 is a norm iteration
-  if (p.norm_every > 0) {
-    const uint64_t ne = (uint64_t)p.norm_every;
-    const uint64_t first = ((k + ne - 1) / ne) * ne;
-    if (first < k + T) nl = (int)(first - k) + 1;
-  }
-  double acc = 0.0;
-  if (nl == 0) {
-    t_body<T, 0>(p, k, par, ring, full, empty);
-  } else if (nl == 1) {
-    acc = t_body<T, 1>(p, k, par, ring, full, empty);
-  } else if (nl == 2) {
-    if constexpr (T >= 2) acc = t_body<T, 2>(p, k, par, ring, full, empty);
-  } else if (nl == 3) {
-    if constexpr (T >= 3) acc = t_body<T, 3>(p, k, par, ring, full, empty);
-  } else {
-    if constexpr (T >= 4) acc = t_body<T, 4>(p, k, par, ring, full, empty);
-  }
-  if (nl > 0) {
-    const double t = block_sum(acc, smem);
-    if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    const unsigned t = atomicAdd(p.done, 1u);
-    s_last = (t == gridDim.x - 1);
-  }
-  __syncthreads();
-  if (s_last) {
-    __threadfence();
-    finish_iteration(p, nl > 0, smem, T);
-  }
+size_t multistep_smem_bytes(int consumers, int stages, int ghosts) {
+  // [full mbarriers][empty mbarriers] padded to 128 B, then the row ring (4G halo floats per side)
+  return (size_t)((32 * stages + 127) / 128) * 128 + (size_t)stages * (4 * consumers + 8 * ghosts) * sizeof(float);
 }
 
 int launch_jacobi_t(const JacobiParams& p, int grid, int block, int T, cudaStream_t s) {
-  const size_t smem = staged_smem_bytes(p.consumers, p.stages);
+  const size_t smem = multistep_smem_bytes(p.consumers, p.stages, p.ghosts);
+  if (p.ghosts == 2) return launch_jacobi_t_g2(p, grid, block, T, smem, s);
+  if (p.ghosts != 1) return fail(UC_ERR_ARG, "%d ghost lanes per warp side not in 1..2", p.ghosts);
   switch (T) {
-    case 1: jacobi_t_kernel<1><<<grid, block, smem, s>>>(p); break;
-    case 2: jacobi_t_kernel<2><<<grid, block, smem, s>>>(p); break;
-    case 3: jacobi_t_kernel<3><<<grid, block, smem, s>>>(p); break;
-    case 4: jacobi_t_kernel<4><<<grid, block, smem, s>>>(p); break;
-    default: return fail(UC_ERR_ARG, "T = %d iterations per launch not in 1..4", T);
+    case 1: jacobi_t_kernel<1, 1><<<grid, block, smem, s>>>(p); break;
+    case 2: jacobi_t_kernel<2, 1><<<grid, block, smem, s>>>(p); break;
+    case 3: jacobi_t_kernel<3, 1><<<grid, block, smem, s>>>(p); break;
+    case 4: jacobi_t_kernel<4, 1><<<grid, block, smem, s>>>(p); break;
+    default: return fail(UC_ERR_ARG, "T = %d iterations per launch not in 1..4 (one ghost lane)", T);
   }
   UC_CUDA(cudaGetLastError());
   return UC_OK;
 }
 
 int preload_multistep() {
-  const void* fns[] = {(const void*)jacobi_t_kernel<1>, (const void*)jacobi_t_kernel<2>,
-                       (const void*)jacobi_t_kernel<3>, (const void*)jacobi_t_kernel<4>};
+  const void* fns[] = {(const void*)jacobi_t_kernel<1, 1>, (const void*)jacobi_t_kernel<2, 1>,
+                       (const void*)jacobi_t_kernel<3, 1>, (const void*)jacobi_t_kernel<4, 1>};
   for (const void* f : fns) {
     UC_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
     cudaFuncAttributes a;
     UC_CUDA(cudaFuncGetAttributes(&a, f));
   }
-  return UC_OK;
+  return preload_multistep_g2();
 }
 
-int multistep_occupancy(int block, size_t smem, int* blocks_per_sm) {
-  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_t_kernel<4>, block, smem));
+int multistep_max_consumers(int ghosts) { return ghosts == 2 ? kMaxBlockG2 : kMaxBlock; }
+
+int multistep_occupancy(int block, size_t smem, int ghosts, int* blocks_per_sm) {
+  if (ghosts == 2) return multistep_occupancy_g2(block, smem, blocks_per_sm);
+  UC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, jacobi_t_kernel<4, 1>, block, smem));
   return UC_OK;
 }
 

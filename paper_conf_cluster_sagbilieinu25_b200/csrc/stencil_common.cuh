@@ -43,6 +43,16 @@ constexpr int kTwoStepUnroll = UC_TWO_STEP_UNROLL;
 #ifndef UC_T_MINBLOCKS
 #define UC_T_MINBLOCKS 2
 #endif
+// the same for the two-ghost-lane layout (T up to 8: twice the register window, 165 registers at
+// T = 8): one block per SM of up to UC_T8_MAXTHREADS threads (12 warps: 3 per SM sub-partition,
+// so the 16K-register file of a sub-partition allows 170 registers per thread)
+#ifndef UC_T8_MINBLOCKS
+#define UC_T8_MINBLOCKS 2
+#endif
+#ifndef UC_T8_MAXTHREADS
+#define UC_T8_MAXTHREADS 256
+#endif
+constexpr int kMaxBlockG2 = UC_T8_MAXTHREADS - 32;  // consumer threads per block, two ghost lanes
 #ifndef UC_T_UNROLL
 #define UC_T_UNROLL 3
 #endif

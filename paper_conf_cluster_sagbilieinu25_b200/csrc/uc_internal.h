@@ -68,6 +68,7 @@ struct JacobiParams {
   int tile_rows;                       // variant 2: rows per work item
   int strip4;                          // variant 5: owned float4 columns per strip (ghost-lane layout)
   int chunk_shrink;                    // variant 5: rows taken off the first/last row chunk
+  int ghosts;                          // variant 5: ghost lanes per warp side (1: T <= 4, 2: T <= 8)
   double* partials;                    // local [grid] per-block partial sums
   double* rank_sum;                    // local: this rank's sum of squares (host-mode allreduce in place)
   double* norm_hist;                   // local: norms by round m (ring of norm_cap)
@@ -105,7 +106,17 @@ int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStre
 int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_t(const JacobiParams& p, int grid, int block, int T, cudaStream_t s);
 int preload_multistep();                                             // multistep.cu
-int multistep_occupancy(int block, size_t smem, int* blocks_per_sm); // the deepest instance bounds all T
+// the deepest instance of a ghost layout (G = 1: T = 4; G = 2: T = 8) bounds the geometry of all T
+int multistep_occupancy(int block, size_t smem, int ghosts, int* blocks_per_sm);
+size_t multistep_smem_bytes(int consumers, int stages, int ghosts);  // the ring carries 4G halo floats per side
+int launch_jacobi_t_g2(const JacobiParams& p, int grid, int block, int T, size_t smem, cudaStream_t s);  // multistep_g2.cu
+int preload_multistep_g2();
+int launch_jacobi_t_g2b(const JacobiParams& p, int grid, int block, int T, size_t smem, cudaStream_t s);  // multistep_g2b.cu
+int preload_multistep_g2b();
+int launch_jacobi_t_g2c(const JacobiParams& p, int grid, int block, size_t smem, cudaStream_t s);  // multistep_g2c.cu
+int preload_multistep_g2c();
+int multistep_occupancy_g2(int block, size_t smem, int* blocks_per_sm);
+int multistep_max_consumers(int ghosts);  // consumer threads per block the launch bounds allow
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
@@ -223,6 +234,7 @@ struct uc_jacobi {
   int levels = 1;                // variant 5: iterations per launch T
   int strip4 = 0;                // variant 5: owned float4 columns per strip
   int chunk_shrink = 0;          // variant 5: rows taken off the first/last row chunk
+  int ghosts = 1;                // variant 5: ghost lanes per warp side (2 when T > 4)
   size_t slab_elems = 0;
   int strips = 0;               // current column strips (launch geometry)
   int max_strips = 0;           // flag capacity per side = ceil(nx/4 / 32)

@@ -14,6 +14,6 @@ tail -3 $OUT/bench.txt
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
   --log-file $OUT/launches.csv python bench.py --steps 2 --warmup 3 --no-extras > $OUT/launches_bench.txt 2>&1
 echo "launches rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:jacobi_t_kernel -s 80 -c 2 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:jacobi_t_kernel -s 80 -c 1 \
   -o $OUT/prof python bench.py --steps 1 --warmup 3 --no-extras > $OUT/prof_bench.txt 2>&1
 echo "full rc=$?"

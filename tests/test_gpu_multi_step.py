@@ -1,5 +1,6 @@
-"""GPU parity of kernel variant 5 (T = 1..4 Jacobi iterations per launch, temporal blocking of
-depth T, ghost-lane layout) against the CPU oracle.
+"""GPU parity of kernel variant 5 (T = 1..8 Jacobi iterations per launch, temporal blocking of
+depth T, ghost-lane layout: one ghost lane per warp side for T <= 4, two for T = 5..8) against
+the CPU oracle.
 
 Variant 5 keeps A_{k+1}..A_{k+T-1} in registers and stores only A_{k+T}; the boundary rows of
 every intermediate iterate are still exchanged with the neighbours (rounds 1..T per launch).
@@ -15,7 +16,8 @@ from test_gpu_jacobi import NORM_RTOL, _check, _oracle
 
 pytestmark = pytest.mark.gpu
 
-TS = [1, 2, 3, 4]
+TS = [1, 2, 3, 4, 5, 6, 7, 8]
+TG = [2, 3, 4, 6, 8]  # both ghost layouts
 
 
 def _v5(T, **kw):
@@ -31,7 +33,7 @@ def test_c1_256(T, topology, iters, ne):
     assert res["launch"]["variant"] == 5 and res["launch"]["tile_rows"] == T
 
 
-@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("T", TG)
 @pytest.mark.parametrize("nx,ny,iters", [(4, 8, 9), (8, 9, 20), (12, 16, 9), (1028, 64, 38), (2052, 33, 13),
                                          (4096, 40, 8), (36, 8, 12), (40, 9, 11), (964, 30, 17)])
 @pytest.mark.parametrize("topology", ["ring", "dirichlet"])
@@ -40,7 +42,7 @@ def test_shapes_single_rank(T, nx, ny, iters, topology):
     _check(nx, ny, 1, topology, "device", iters, norm_every=4, **_v5(T))
 
 
-@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("T", TG)
 @pytest.mark.parametrize("P", [2, 3, 4, 8])
 @pytest.mark.parametrize("topology", ["ring", "dirichlet"])
 def test_partition_invariance(T, P, topology):
@@ -48,24 +50,26 @@ def test_partition_invariance(T, P, topology):
     _check(520, 24 * P, P, topology, "device", 27, norm_every=5, **_v5(T))
 
 
-@pytest.mark.parametrize("T", [2, 3, 4])
-@pytest.mark.parametrize("P,ny", [(2, 4), (2, 6), (3, 9), (2, 8), (4, 32), (2, 16)])
+@pytest.mark.parametrize("T", [2, 3, 4, 5, 8])
+@pytest.mark.parametrize("P,ny", [(2, 4), (2, 6), (3, 9), (2, 8), (4, 32), (2, 16), (2, 30)])
 def test_few_rows_per_rank(T, P, ny):
     """n = 2..8: launches shrink to the deepest T' with n >= 2T'; one row chunk per strip."""
     for topology in ("ring", "dirichlet"):
         _check(64, ny, P, topology, "device", 13, norm_every=0, **_v5(T))
 
 
-@pytest.mark.parametrize("T", [2, 4])
+@pytest.mark.parametrize("T", [2, 4, 6, 8])
 @pytest.mark.parametrize("block_x,bps,stages", [(32, 1, 3), (64, 2, 4), (128, 0, 2), (256, 1, 8), (96, 0, 5)])
 def test_launch_geometries(T, block_x, bps, stages):
     """Strip width (ghost lanes meet strip edges), chunk count and ring depth: 4 ranks."""
+    if T > 4:  # two ghost lanes: the launch bounds allow 7 consumer warps per block
+        block_x = min(block_x, 224)
     res = _check(1028, 128, 4, "ring", "device", 12, norm_every=4, block_x=block_x, blocks_per_sm=bps,
                  stages=stages, **_v5(T))
     assert res["launch"]["variant"] == 5
 
 
-@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("T", TG)
 def test_random_values_everywhere(T):
     nx, ny = 1028, 48
     rng = np.random.default_rng(11)
@@ -76,7 +80,7 @@ def test_random_values_everywhere(T):
     _check(nx, ny, 2, "dirichlet", "device", 14, norm_every=0, init=init, **_v5(T))
 
 
-@pytest.mark.parametrize("T", [3, 4])
+@pytest.mark.parametrize("T", [3, 4, 8])
 def test_graph_eager_stepwise_chunked_agree(T):
     kw = _v5(T)
     a = solve_gpu(516, 64, 2, "ring", "device", 30, 7, use_graph=True, **kw)
@@ -112,7 +116,7 @@ def test_switch_variants_and_modes_mid_run():
         coord.set_timeout(5.0)
         J = U.Jacobi(comm, nx, ny)
         out = []
-        for v, T, it in ((5, 4, 10), (4, 0, 5), (5, 3, 7), (1, 0, 3), (5, 4, 9)):
+        for v, T, it in ((5, 4, 10), (4, 0, 5), (5, 3, 7), (1, 0, 3), (5, 8, 19), (5, 6, 8), (5, 4, 9)):
             J.set_launch(v, 0, 0, 0, T)
             out.append(J.run(coord, it, 5))
             coord.sync()
@@ -125,7 +129,7 @@ def test_switch_variants_and_modes_mid_run():
         return slab, np.concatenate(out)
 
     res = run_ranks(P, body)
-    _, want, want_norms = _oracle(nx, ny, "ring", 34, 5)
+    _, want, want_norms = _oracle(nx, ny, "ring", 61, 5)
     assert_slabs_equal_global([r[0] for r in res], want, P, "ring")
     assert np.allclose(res[0][1], want_norms, rtol=NORM_RTOL, atol=0)
 
@@ -148,23 +152,25 @@ def test_switch_variants_and_modes_mid_run():
     assert_slabs_equal_global([out], want, 1, "ring")
 
 
+@pytest.mark.parametrize("T", [4, 8])
 @pytest.mark.parametrize("mode", ["host", "partial"])
-def test_host_and_partial_modes(mode):
-    _check(1028, 40, 1, "ring", mode, 11, norm_every=3, **_v5(4))
+def test_host_and_partial_modes(mode, T):
+    _check(1028, 40, 1, "ring", mode, 11, norm_every=3, **_v5(T))
 
 
-def test_subnormal_front_no_ftz():
-    nx, ny = 96, 8
+@pytest.mark.parametrize("T", [4, 8])
+def test_subnormal_front_no_ftz(T):
+    nx, ny = 96, 16
     a = np.zeros((ny + 2, nx), np.float32)
     a[:, 0] = 1.0
     for k in (64, 70, 74, 75):
-        res = solve_gpu(nx, ny, 1, "ring", "device", k, 0, init=a, **_v5(4))
+        res = solve_gpu(nx, ny, 1, "ring", "device", k, 0, init=a, **_v5(T))
         s = res["final"][0]
         want = np.float32(2.0 ** (-2 * k)) if k <= 74 else np.float32(0.0)
         assert s[1, k] == want and s[1, k + 1] == 0.0
 
 
-@pytest.mark.parametrize("T", [2, 3, 4])
+@pytest.mark.parametrize("T", [2, 3, 4, 6, 8])
 def test_full_size_16384(T):
     """16384^2 (configs[2]/[3] at P = 1): whole grid bit-exact, norms on every level."""
     _check(16384, 16384, 1, "ring", "device", 2 * T + 1, norm_every=T, **_v5(T))
@@ -174,5 +180,6 @@ def test_config2_strong_16384_over_8_ranks():
     _check(16384, 16384, 8, "ring", "device", 9, norm_every=4, **_v5(4))
 
 
-def test_config1_4096_2ranks_1000_iterations():
-    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, **_v5(4))
+@pytest.mark.parametrize("T", [4, 8])
+def test_config1_4096_2ranks_1000_iterations(T):
+    _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, **_v5(T))

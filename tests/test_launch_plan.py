@@ -27,7 +27,7 @@ def restated(variant, levels, mode, n, iters, ne):
     return [1] * iters
 
 
-CASES = list(itertools.product([1, 4, 5], [1, 2, 3, 4], [DEV, HOST, PARTIAL], [1, 2, 3, 4, 7, 8, 16384]))
+CASES = list(itertools.product([1, 4, 5], [1, 2, 3, 4, 6, 8], [DEV, HOST, PARTIAL], [1, 2, 3, 4, 7, 8, 15, 16, 16384]))
 
 
 @pytest.mark.parametrize("variant,levels,mode,n", CASES)
@@ -61,10 +61,13 @@ def test_bench_configuration_plan():
     assert U.launch_plan(5, 4, DEV, 16384, 10, 3) == [3, 3, 3, 1]   # norm every 3 < T
     assert U.launch_plan(5, 4, HOST, 16384, 3, 0) == [1, 1, 1]
     assert U.launch_plan(4, 0, DEV, 16384, 5, 0) == [2, 2, 1]
+    # two ghost lanes (T up to 8): 100 = 12 x 8 + 4
+    assert U.launch_plan(5, 8, DEV, 16384, 100, 100) == [8] * 12 + [4]
+    assert U.launch_plan(5, 8, DEV, 10, 100, 0) == [5] * 20           # n = 10: T' = 5
 
 
 def test_plan_argument_errors():
     with pytest.raises(U.UCError):
-        U.launch_plan(5, 5, DEV, 100, 10, 0)
+        U.launch_plan(5, 9, DEV, 100, 10, 0)
     with pytest.raises(U.UCError):
         U.launch_plan(5, 4, DEV, 0, 10, 0)
