@@ -60,6 +60,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     if not force and not defines and out is None and not _stale():
         if any(not os.path.exists(t) or os.path.getmtime(t) < os.path.getmtime(s) for s, t in _example_targets()):
             build_examples()
+        build_native()
         return LIB
     nd = nccl_dir()
     os.makedirs(os.path.dirname(os.path.abspath(target)), exist_ok=True)
@@ -92,6 +93,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     os.replace(tmp, target)
     if out is None:
         build_examples()
+        build_native()
     return target
 
 
@@ -101,6 +103,24 @@ def _example_targets():
     t += [(s, os.path.join(ex, "lib" + os.path.basename(s)[:-3].replace("device_api_ring", "uc_device_example") + ".so"))
           for s in glob.glob(os.path.join(ex, "*.cu"))]
     return t
+
+
+NATIVE = os.path.join(ROOT, "benchmarks", "native")
+
+
+def build_native(force: bool = False) -> str:
+    """In-box comparator (not the product): the Listing-3 Jacobi on NCCL's device
+    API, benchmarks/native/nccl_dev_jacobi.cu -> libuc_nccl_dev.so (nvcc sm_100a, the wheel's NCCL)."""
+    src = os.path.join(NATIVE, "nccl_dev_jacobi.cu")
+    out = os.path.join(NATIVE, "libuc_nccl_dev.so")
+    deps = [src, os.path.join(NATIVE, "nccl_dev_jacobi.h"), __file__]
+    if not force and os.path.exists(out) and all(os.path.getmtime(d) <= os.path.getmtime(out) for d in deps):
+        return out
+    nd = nccl_dir()
+    subprocess.check_call([nvcc(), *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
+                           "-I", os.path.join(nd, "include"), src, "-o", out, "-L", os.path.join(nd, "lib"),
+                           "-l:libnccl.so.2", "-Xlinker", "-rpath=" + os.path.join(nd, "lib")])
+    return out
 
 
 def build_examples() -> None:

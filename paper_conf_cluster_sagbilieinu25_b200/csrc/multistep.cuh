@@ -199,18 +199,25 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
 // The producer streams the A_k rows a-T..b+T; consumers keep two rows per level.
 // One row of the T-level march: take the next A_k row from the ring, advance every level, store
 // the A_{k+T} row (STORE: from the 2T-th row on).
-template <int T, int NL, bool DIRI, bool STORE>
-__device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
-                                       const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
-                                       float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+// Take the next A_k row from the ring (wait for its stage, read it, release the stage).
+__device__ __forceinline__ float4 t_fetch(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
+                                          const GhostLayout& g, RingCursor& cur) {
   mbar_wait(full + cur.st, cur.ph);
-  float4 nv = *reinterpret_cast<const float4*>(ring + (size_t)cur.st * ST + g.ring_off);
+  const float4 nv = *reinterpret_cast<const float4*>(ring + (size_t)cur.st * ST + g.ring_off);
   __syncwarp();
   mbar_arrive_if(empty + cur.st, (threadIdx.x & 31) == 0);
   if (++cur.st == NS) {
     cur.st = 0;
     cur.ph ^= 1u;
   }
+  return nv;
+}
+
+// Advance every level by the A_k row nv (the i-th row of the march) and store the A_{k+T} row
+// (STORE: from the 2T-th row on).
+template <int T, int NL, bool DIRI, bool STORE>
+__device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx4, int a, int b, int i,
+                                         float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
 #pragma unroll
   for (int j = 0; j < T; ++j) {
     const float4 o = row_update_g<DIRI>(w0[j], w1[j], nv, g.x4, nx4);  // level j+1, row r-j-1
@@ -226,6 +233,15 @@ __device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64
     if (g.own) st4(out, nv);
     out += pitch;
   }
+}
+
+// One row of the T-level march: fetch the next A_k row, advance every level, store.
+template <int T, int NL, bool DIRI, bool STORE>
+__device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
+                                       const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
+                                       float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+  const float4 nv = t_fetch(ring, full, empty, ST, NS, g, cur);
+  t_levels<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, out, pitch, acc);
 }
 
 template <int T, int NL, bool DIRI, int G>
