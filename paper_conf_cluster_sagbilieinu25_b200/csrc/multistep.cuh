@@ -54,10 +54,10 @@ __device__ __forceinline__ void quarter2_rn(float a0, float a1, float& r0, float
 
 // row_update for the ghost-lane layout (no cross-warp operand): new = 0.25f*((l+r)+(t+b)) with
 // the vertical sums t+b, the outer sums and the products packed two columns per instruction.
+// L, R: the left neighbour of column 4*x4 and the right neighbour of column 4*x4+3 (the
+// adjacent lanes' c.w and c.x).
 template <bool DIRI = true>
-__device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, int x4, int nx4) {
-  const float L = __shfl_up_sync(kFull, c.w, 1);    // lane 0: its own value (ghost lane, discarded)
-  const float R = __shfl_down_sync(kFull, c.x, 1);  // lane 31: likewise
+__device__ __forceinline__ float4 row_update_lr(float4 up, float4 c, float4 dn, float L, float R, int x4, int nx4) {
 #if UC_PACKED_F32X2
   const float hx = __fadd_rn(L, c.y), hy = __fadd_rn(c.x, c.z);
   const float hz = __fadd_rn(c.y, c.w), hw = __fadd_rn(c.z, R);
@@ -81,6 +81,12 @@ __device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, i
   o.w = (x4 == nx4 - 1) ? c.w : upd(c.z, R, up.w, dn.w);
 #endif
   return o;
+}
+template <bool DIRI = true>
+__device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, int x4, int nx4) {
+  const float L = __shfl_up_sync(kFull, c.w, 1);    // lane 0: its own value (ghost lane, discarded)
+  const float R = __shfl_down_sync(kFull, c.x, 1);  // lane 31: likewise
+  return row_update_lr<DIRI>(up, c, dn, L, R, x4, nx4);
 }
 
 struct GhostLayout {
@@ -215,12 +221,24 @@ __device__ __forceinline__ float4 t_fetch(const float* ring, uint64_t* full, uin
 
 // Advance every level by the A_k row nv (the i-th row of the march) and store the A_{k+T} row
 // (STORE: from the 2T-th row on).
-template <int T, int NL, bool DIRI, bool STORE>
-__device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx4, int a, int b, int i,
-                                         float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+// The horizontal neighbours of every level's middle row (w1[j], known before the step's new row
+// arrives): shuffled up front, off the level chain (new row -> level 1 -> ... -> level T).
+template <int T>
+__device__ __forceinline__ void t_neighbours(const float4 (&w1)[T], float (&L)[T], float (&R)[T]) {
 #pragma unroll
   for (int j = 0; j < T; ++j) {
-    const float4 o = row_update_g<DIRI>(w0[j], w1[j], nv, g.x4, nx4);  // level j+1, row r-j-1
+    L[j] = __shfl_up_sync(kFull, w1[j].w, 1);    // lane 0: its own value (ghost lane, discarded)
+    R[j] = __shfl_down_sync(kFull, w1[j].x, 1);  // lane 31: likewise
+  }
+}
+
+template <int T, int NL, bool DIRI, bool STORE>
+__device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx4, int a, int b, int i,
+                                         float4 (&w0)[T], float4 (&w1)[T], const float (&L)[T], const float (&R)[T],
+                                         float*& out, size_t pitch, double& acc) {
+#pragma unroll
+  for (int j = 0; j < T; ++j) {
+    const float4 o = row_update_lr<DIRI>(w0[j], w1[j], nv, L[j], R[j], g.x4, nx4);  // level j+1, row r-j-1
     if (NL == j + 1 && g.own) {
       const int y = a - T + i - j - 1;
       if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
@@ -235,13 +253,22 @@ __device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx
   }
 }
 
+// Shuffle the neighbours of the next step before its ring wait (HOIST) or after it.  Measured per
+// instance (profiles/r1_t8_sweep.txt, pass 7): hoisting gains 2-8 % at T = 4, 5, 7, 8 and loses
+// 2.5 % at T = 6 with two ghost lanes, whose 128 registers are exactly the cap.
+template <int T, int G>
+constexpr bool kHoistNeighbours = !(T == 6 && G == 2);
+
 // One row of the T-level march: fetch the next A_k row, advance every level, store.
-template <int T, int NL, bool DIRI, bool STORE>
+template <int T, int NL, bool DIRI, bool STORE, bool HOIST>
 __device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
                                        const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
                                        float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+  float L[T], R[T];
+  if constexpr (HOIST) t_neighbours<T>(w1, L, R);  // overlaps the ring wait and the shared-memory load
   const float4 nv = t_fetch(ring, full, empty, ST, NS, g, cur);
-  t_levels<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, out, pitch, acc);
+  if constexpr (!HOIST) t_neighbours<T>(w1, L, R);
+  t_levels<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, L, R, out, pitch, acc);
 }
 
 template <int T, int NL, bool DIRI, int G>
@@ -290,10 +317,12 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
   // the first 2T rows only fill the levels (rows >= 2T + 1 since a <= b)
 #pragma unroll
   for (int i = 0; i < 2 * T; ++i)
-    t_step<T, NL, DIRI, false>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc);
+    t_step<T, NL, DIRI, false, kHoistNeighbours<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
+                                                      pitch, acc);
 #pragma unroll(kTUnroll)
   for (int i = 2 * T; i < rows; ++i)
-    t_step<T, NL, DIRI, true>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc);
+    t_step<T, NL, DIRI, true, kHoistNeighbours<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
+                                                     pitch, acc);
 }
 
 template <int T, int NL, int G>

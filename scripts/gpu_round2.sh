@@ -17,3 +17,9 @@ echo "launches rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:jacobi_t_kernel -s 80 -c 1 \
   -o $OUT/prof python bench.py --steps 1 --warmup 3 --no-extras > $OUT/prof_bench.txt 2>&1
 echo "full rc=$?"
+# the N > 1 launch path (torchrun, one process per rank, CUDA IPC peers) on the one GPU of the box
+timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 \
+  bench.py --gpus 2 --same-device --steps 3 --warmup 3 --ny-per-gpu 8192 > $OUT/bench_2proc.txt 2>&1; echo "2proc rc=$?" >> $OUT/bench_2proc.txt
+tail -2 $OUT/bench_2proc.txt | cut -c1-600
+timeout 300 python bench.py --impl reference --steps 2 --warmup 3 > $OUT/bench_ref.txt 2>&1; echo "ref rc=$?" >> $OUT/bench_ref.txt
+tail -2 $OUT/bench_ref.txt | cut -c1-600
