@@ -53,8 +53,6 @@ struct CGParams {
   unsigned int* err;
 };
 
-constexpr int kTPR = 8;  // lanes per CSR row in the SpMV
-
 __device__ __forceinline__ double cg_block_sum(double v, double* smem) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);

@@ -23,3 +23,6 @@ timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --mast
 tail -2 $OUT/bench_2proc.txt | cut -c1-600
 timeout 300 python bench.py --impl reference --steps 2 --warmup 3 > $OUT/bench_ref.txt 2>&1; echo "ref rc=$?" >> $OUT/bench_ref.txt
 tail -2 $OUT/bench_ref.txt | cut -c1-600
+# configs[2]'s per-GPU share at P = 8 (16384 x 2048 slab) on one GPU, with the halo leg
+timeout 300 python bench.py --steps 10 --warmup 3 --ny-per-gpu 2048 --halo-only > $OUT/bench_slab2048.txt 2>&1; echo "slab rc=$?" >> $OUT/bench_slab2048.txt
+tail -2 $OUT/bench_slab2048.txt | cut -c1-300
