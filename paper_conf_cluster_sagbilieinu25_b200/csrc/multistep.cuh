@@ -257,10 +257,10 @@ __device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx
 // instance (profiles/r1_t8_sweep.txt, pass 7): hoisting gains 2-8 % at T = 4, 5, 7, 8 and loses
 // 2.5 % at T = 6 with two ghost lanes, whose 128 registers are exactly the cap.
 #ifndef UC_HOIST_ALL
-#define UC_HOIST_ALL 0  // A/B knob: hoist on every instance
+#define UC_HOIST_ALL 0  // A/B knob: 1 = hoist on every instance, -1 = on none
 #endif
 template <int T, int G>
-constexpr bool kHoistNeighbours = UC_HOIST_ALL || !(T == 6 && G == 2);
+constexpr bool kHoistNeighbours = UC_HOIST_ALL == 1 || (UC_HOIST_ALL == 0 && !(T == 6 && G == 2));
 
 // One row of the T-level march: fetch the next A_k row, advance every level, store.
 template <int T, int NL, bool DIRI, bool STORE, bool HOIST>
