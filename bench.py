@@ -228,7 +228,7 @@ def run_ours(a):
     use_graph = not a.no_graph
     ips = a.iters_per_step
     pts_rank = n * (nx - 2)
-    norms_buf = U.pinned_f64(max(1, ips // max(1, a.norm_every) + 1))
+    norms_buf = np.zeros(max(1, ips // max(1, a.norm_every) + 1), np.float64)
 
     def step():
         J.run(coord, ips, a.norm_every, use_graph, norms_out=norms_buf)
@@ -276,7 +276,7 @@ def run_ours(a):
     # ---------------- dominant kernel: per-launch events around single launches (no norm / norm)
     def kernel_ms(compute_norm, reps, iters_per_launch):
         es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
-        buf = U.pinned_f64(2)
+        buf = np.zeros(2, np.float64)
         for s, e in es:
             s.record(stream)
             if iters_per_launch > 1:  # one multi-iteration launch (norm_every = T: one norm round in it)

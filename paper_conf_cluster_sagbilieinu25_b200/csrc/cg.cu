@@ -296,6 +296,7 @@ struct uc_cg {
   double* partials = nullptr;
   unsigned int* done = nullptr;
   double* hist = nullptr;
+  double* hist_stage = nullptr;  // page-locked mirror of hist for pageable outputs
   int hist_cap = 65536;
   int grid = 0, spmv_grid = 0, partials_cap = 0;
   // SpMV: lanes per row, rows in flight per lane group.  Round-1 sweep at 160^3, 27-point
@@ -446,6 +447,7 @@ int uc_cg_create(uc_comm* c, int nx, int ny, int nz, int stencil, uint64_t seed,
     cudaFree(cg->partials);
     cudaFree(cg->done);
     cudaFree(cg->hist);
+    if (cg->hist_stage) cudaFreeHost(cg->hist_stage);
     if (cg->aux) cudaStreamDestroy(cg->aux);
     delete cg;
     return rc;
@@ -496,6 +498,7 @@ int uc_cg_create(uc_comm* c, int nx, int ny, int nz, int stencil, uint64_t seed,
   if (e == cudaSuccess) e = cudaMalloc(&cg->st, sizeof(CGState));
   if (e == cudaSuccess) e = cudaMalloc(&cg->done, sizeof(unsigned int));
   if (e == cudaSuccess) e = cudaMalloc(&cg->hist, sizeof(double) * cg->hist_cap);
+  if (e == cudaSuccess) e = cudaHostAlloc((void**)&cg->hist_stage, sizeof(double) * cg->hist_cap, cudaHostAllocDefault);
   if (e != cudaSuccess) return bail(fail(UC_ERR_OOM, "CG state: %s", cudaGetErrorString(e)));
   CGState st0{rr0, 0.0, 0.0, 0.0, 0ull, 0ull};
   cudaStream_t s = cg->aux;
@@ -568,8 +571,7 @@ int uc_cg_run(uc_coord* k, uc_cg* cg, int iters, double* rr_out, int use_graph) 
     while (done < iters) {
       const int idx = (int)((k0 + done) % cg->hist_cap);
       const int len = std::min(iters - done, cg->hist_cap - idx);
-      UC_CUDA(cudaMemcpyAsync(rr_out + done, cg->hist + idx, sizeof(double) * len, cudaMemcpyDeviceToHost,
-                              k->stream));
+      UC_TRY(enqueue_d2h_f64(k, rr_out + done, cg->hist + idx, cg->hist_stage + idx, (size_t)len));
       done += len;
     }
   }
@@ -621,6 +623,7 @@ int uc_cg_destroy(uc_cg* cg) {
   cudaFree(cg->partials);
   cudaFree(cg->done);
   cudaFree(cg->hist);
+  if (cg->hist_stage) cudaFreeHost(cg->hist_stage);
   cudaStreamDestroy(cg->aux);
   c->live_objects--;
   delete cg;

@@ -28,6 +28,27 @@ int fail(int status, const char* fmt, ...) {
   return status;
 }
 
+int enqueue_d2h_f64(uc_coord* k, double* host, const double* dev, double* stage, size_t n) {
+  if (!host || n == 0) return UC_OK;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  UC_CUDA(cudaStreamIsCapturing(k->stream, &cs));
+  cudaPointerAttributes a{};
+  const bool pinned = cudaPointerGetAttributes(&a, host) == cudaSuccess && a.type != cudaMemoryTypeUnregistered;
+  cudaGetLastError();  // clear a failed query
+  if (pinned || !stage || cs != cudaStreamCaptureStatusNone) {
+    UC_CUDA(cudaMemcpyAsync(host, dev, n * sizeof(double), cudaMemcpyDeviceToHost, k->stream));
+    return UC_OK;
+  }
+  UC_CUDA(cudaMemcpyAsync(stage, dev, n * sizeof(double), cudaMemcpyDeviceToHost, k->stream));
+  k->pending.push_back({host, stage, n});
+  return UC_OK;
+}
+
+static void flush_pending(uc_coord* k) {
+  for (const auto& c : k->pending) memcpy(c.dst, c.src, c.n * sizeof(double));
+  k->pending.clear();
+}
+
 static uint64_t host_hash() {
   std::string id;
   char name[256] = {0};
@@ -409,7 +430,7 @@ int uc_coord_destroy(uc_coord* k) {
   if (!k) return fail(UC_ERR_ARG, "coord is NULL");
   if (k->live_jacobi_users) return fail(UC_ERR_STATE, "coordinator still in use");
   UC_CUDA(cudaSetDevice(k->comm->env->device));
-  cudaStreamSynchronize(k->stream);
+  if (cudaStreamSynchronize(k->stream) == cudaSuccess) flush_pending(k);
   if (k->nccl) ncclCommDestroy(k->nccl);
   if (k->ar_scratch) UC_TRY(uc_mem_free_symmetric(k->ar_scratch));
   if (k->coll_flags) UC_TRY(uc_mem_free_symmetric(k->coll_flags));
@@ -425,6 +446,7 @@ int uc_coord_sync(uc_coord* k) {
   if (!k) return fail(UC_ERR_ARG, "coord is NULL");
   UC_CUDA(cudaSetDevice(k->comm->env->device));
   UC_CUDA(cudaStreamSynchronize(k->stream));
+  flush_pending(k);
   unsigned int err = 0;
   UC_CUDA(cudaMemcpy(&err, k->err, sizeof err, cudaMemcpyDeviceToHost));
   if (err) {

@@ -118,6 +118,15 @@ int preload_multistep_g2c();
 int multistep_occupancy_g2(int block, size_t smem, int* blocks_per_sm);
 int multistep_max_consumers(int ghosts);  // consumer threads per block the launch bounds allow
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
+// Stream-ordered device -> host copy of n doubles on the coordinator's stream that never blocks
+// the calling thread: into page-locked memory directly; into pageable memory into `stage`
+// (page-locked, >= n doubles, owned by the caller) and from there into `host` at the next
+// uc_coord_sync / uc_coord_destroy (the outputs' contract: valid after uc_coord_sync).  A plain
+// pageable cudaMemcpyAsync returns only after the stream's earlier work, and with several ranks
+// in one process that wait can stall a peer's launch behind a kernel waiting for that peer; a
+// stream host function instead serialises on the driver's callback thread across streams.
+// Inside a stream capture: a plain cudaMemcpyAsync.
+int enqueue_d2h_f64(uc_coord* k, double* host, const double* dev, double* stage, size_t n);
 int launch_norm_finish(double* rank_sum, double* norm_hist, int norm_cap, unsigned long long* k_dev,
                        int norm_every, cudaStream_t s);
 int launch_init_field(float* slab0, float* slab1, int nx, int n, int ny, int row0, int ring,
@@ -213,6 +222,12 @@ struct uc_coord {
   uint64_t p2p_epoch[3][UC_MAX_RANKS] = {};  // signal base of the next uc_p2p_bench call, per (pattern, peer)
   unsigned int* p2p_bar = nullptr;     // grid barrier [count, gen] of the p2p kernel
   int live_jacobi_users = 0;
+  struct PendingCopy {
+    double* dst;
+    const double* src;
+    size_t n;
+  };
+  std::vector<PendingCopy> pending;    // staged pageable outputs, copied at uc_coord_sync
 };
 
 struct JacobiGraph {
@@ -245,6 +260,7 @@ struct uc_jacobi {
   uint64_t* blk_done = nullptr;  // [partials_cap] per-block completed iteration (variant 3)
   double* rank_sum = nullptr;
   double* norm_hist = nullptr;
+  double* norm_stage = nullptr;  // page-locked mirror of norm_hist for pageable norm outputs
   int norm_cap = 4096;
   cudaStream_t aux = nullptr;    // private non-blocking stream (init, synchronous copies)
   int variant = uc::kDefaultVariant, consumers = 0, stages = 0, tile_rows = 0;

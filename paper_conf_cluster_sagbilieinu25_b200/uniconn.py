@@ -24,14 +24,6 @@ from ._lib import (ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, U
                    UCError, check, lib)
 
 
-def pinned_f64(n: int) -> np.ndarray:
-    """A float64 numpy array in page-locked host memory (torch's pinned allocator).  Norm and
-    residual outputs are written by cudaMemcpyAsync on the coordinator's stream; into pageable
-    memory that copy blocks the calling thread inside the driver, which can stall another
-    thread's launch of the kernel this rank's kernel is waiting for (virtual ranks in one process)."""
-    import torch
-    return torch.zeros(max(1, n), dtype=torch.float64, pin_memory=True).numpy()[:n]
-
 
 AllgatherImpl = Callable[[bytes, int], bytes]  # (my bytes, bytes_per_rank) -> size*bytes_per_rank bytes
 
@@ -262,7 +254,7 @@ class CG:
 
     def run(self, coord: Coord, iters: int, use_graph: bool = True,
             rr_out: Optional[np.ndarray] = None) -> np.ndarray:
-        out = rr_out if rr_out is not None else pinned_f64(iters)
+        out = rr_out if rr_out is not None else np.zeros(iters, np.float64)
         check(lib.uc_cg_run(coord.h, self.h, iters, C.c_void_p(out.ctypes.data), int(use_graph)), "uc_cg_run")
         return out[:iters]
 
@@ -307,7 +299,7 @@ class Jacobi:
     def run(self, coord: Coord, iters: int, norm_every: int = 0, use_graph: bool = True,
             norms_out: Optional[np.ndarray] = None) -> np.ndarray:
         cnt = self.num_norms(iters, norm_every)
-        out = norms_out if norms_out is not None else pinned_f64(cnt)
+        out = norms_out if norms_out is not None else np.zeros(cnt, np.float64)
         assert out.size >= cnt and out.dtype == np.float64
         check(lib.uc_jacobi_run(coord.h, self.h, iters, norm_every, C.c_void_p(out.ctypes.data if cnt else None),
                                 int(use_graph)), "uc_jacobi_run")

@@ -44,7 +44,7 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
                 norms = []
                 for i in range(iters):
                     want = norm_every > 0 and J.iteration % norm_every == 0
-                    buf = U.pinned_f64(1)
+                    buf = np.zeros(1, np.float64)
                     J.step(coord, want, buf if want else None)
                     coord.sync()
                     if want:

@@ -299,3 +299,41 @@ def test_config2_strong_16384_over_8_ranks(variant):
 def test_config3_weak_16384_per_rank_2_ranks(variant):
     """BASELINE.json configs[3] at P = 2: 16384 x 32768 global, 16384 x 16384 per rank."""
     _check(16384, 32768, 2, "ring", "device", 4, norm_every=3, variant=variant)
+
+
+def test_pageable_norm_outputs_virtual_ranks():
+    """Norm outputs in pageable numpy memory (staged through page-locked memory and a stream host
+    function, so the copy never blocks a virtual rank's thread): stepwise and run() paths agree
+    with the pinned ones bit for bit."""
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+    from vranks import run_ranks
+    nx, ny, P, iters = 516, 64, 2, 20
+
+    def body(rank, P, ag):
+        env = U.Env(rank, P, 0, ag)
+        comm = U.Comm(env, *U.ring_neighbours(rank, P))
+        st = torch.cuda.Stream()
+        coord = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
+        coord.set_timeout(5.0)
+        J = U.Jacobi(comm, nx, ny)
+        step_norms = np.zeros(iters, np.float64)  # pageable on purpose
+        for i in range(iters):
+            J.step(coord, True, step_norms[i:i + 1])
+        coord.sync()
+        run_norms = np.zeros(iters // 2, np.float64)
+        J.run(coord, iters, 2, False, norms_out=run_norms)
+        coord.sync()
+        comm.barrier()
+        J.destroy()
+        coord.destroy()
+        comm.destroy()
+        env.finalize()
+        return step_norms, run_norms
+
+    res = run_ranks(P, body)
+    _, _, want = _oracle(nx, ny, "ring", 2 * iters, 1)
+    for step_norms, run_norms in res:
+        assert np.allclose(step_norms, want[:iters], rtol=NORM_RTOL, atol=0)
+        assert np.allclose(run_norms, want[iters::2], rtol=NORM_RTOL, atol=0)
