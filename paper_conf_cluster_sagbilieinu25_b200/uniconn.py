@@ -163,9 +163,19 @@ class Coord:
         h = C.c_void_p()
         check(lib.uc_coord_create(comm.h, mode, C.c_void_p(stream), C.byref(h)), "uc_coord_create")
         self.h, self.comm, self.mode, self.stream = h, comm, mode, stream
+        self._outputs = []  # host output arrays the library completes at uc_coord_sync
+
+    def keep(self, arr: np.ndarray) -> np.ndarray:
+        """Hold a host output array alive until the next sync (pageable outputs are written by
+        uc_coord_sync from a page-locked staging copy)."""
+        self._outputs.append(arr)
+        return arr
 
     def sync(self):
-        check(lib.uc_coord_sync(self.h), "uc_coord_sync")
+        try:
+            check(lib.uc_coord_sync(self.h), "uc_coord_sync")
+        finally:
+            self._outputs.clear()
 
     def set_timeout(self, seconds: float):
         check(lib.uc_coord_set_timeout(self.h, int(seconds * 1e9)), "uc_coord_set_timeout")
@@ -233,6 +243,7 @@ class Coord:
         if self.h:
             check(lib.uc_coord_destroy(self.h), "uc_coord_destroy")
             self.h = None
+            self._outputs.clear()
 
 
 def builtin_kernel(name: str) -> int:
@@ -254,7 +265,7 @@ class CG:
 
     def run(self, coord: Coord, iters: int, use_graph: bool = True,
             rr_out: Optional[np.ndarray] = None) -> np.ndarray:
-        out = rr_out if rr_out is not None else np.zeros(iters, np.float64)
+        out = coord.keep(rr_out if rr_out is not None else np.zeros(iters, np.float64))
         check(lib.uc_cg_run(coord.h, self.h, iters, C.c_void_p(out.ctypes.data), int(use_graph)), "uc_cg_run")
         return out[:iters]
 
@@ -290,7 +301,7 @@ class Jacobi:
         return it.value
 
     def step(self, coord: Coord, compute_norm: bool = False, norm_out: Optional[np.ndarray] = None):
-        ptr = norm_out.ctypes.data if norm_out is not None else None
+        ptr = coord.keep(norm_out).ctypes.data if norm_out is not None else None
         check(lib.uc_jacobi_step(coord.h, self.h, int(compute_norm), C.c_void_p(ptr)), "uc_jacobi_step")
 
     def num_norms(self, iters: int, norm_every: int) -> int:
@@ -299,7 +310,7 @@ class Jacobi:
     def run(self, coord: Coord, iters: int, norm_every: int = 0, use_graph: bool = True,
             norms_out: Optional[np.ndarray] = None) -> np.ndarray:
         cnt = self.num_norms(iters, norm_every)
-        out = norms_out if norms_out is not None else np.zeros(cnt, np.float64)
+        out = coord.keep(norms_out if norms_out is not None else np.zeros(cnt, np.float64))
         assert out.size >= cnt and out.dtype == np.float64
         check(lib.uc_jacobi_run(coord.h, self.h, iters, norm_every, C.c_void_p(out.ctypes.data if cnt else None),
                                 int(use_graph)), "uc_jacobi_run")
