@@ -223,10 +223,10 @@ __device__ __forceinline__ float4 t_fetch(const float* ring, uint64_t* full, uin
 // (STORE: from the 2T-th row on).
 // The horizontal neighbours of every level's middle row (w1[j], known before the step's new row
 // arrives): shuffled up front, off the level chain (new row -> level 1 -> ... -> level T).
-template <int T>
+template <int T, int J0 = 0, int J1 = T>
 __device__ __forceinline__ void t_neighbours(const float4 (&w1)[T], float (&L)[T], float (&R)[T]) {
 #pragma unroll
-  for (int j = 0; j < T; ++j) {
+  for (int j = J0; j < J1; ++j) {
     L[j] = __shfl_up_sync(kFull, w1[j].w, 1);    // lane 0: its own value (ghost lane, discarded)
     R[j] = __shfl_down_sync(kFull, w1[j].x, 1);  // lane 31: likewise
   }
@@ -253,24 +253,29 @@ __device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx
   }
 }
 
-// Shuffle the neighbours of the next step before its ring wait (HOIST) or after it.  Measured per
-// instance (profiles/r1_t8_sweep.txt, pass 7): hoisting gains 2-8 % at T = 4, 5, 7, 8 and loses
-// 2.5 % at T = 6 with two ghost lanes, whose 128 registers are exactly the cap.
+// Shuffle the neighbours of the next step's first HOIST levels before its ring wait, the rest
+// after it.  Measured per instance (profiles/r1_t8_sweep.txt, passes 7, 9): hoisting every level
+// gains 2-8 % at T = 4, 5, 7, 8; at <6, 2>, whose 128 registers are exactly the cap, hoisting all
+// six loses 2.5 % and hoisting three gains 1.7 %.
 #ifndef UC_HOIST_ALL
-#define UC_HOIST_ALL 0  // A/B knob: 1 = hoist on every instance, -1 = on none
+#define UC_HOIST_ALL 0  // A/B knob: 1 = hoist every level on every instance, -1 = none
 #endif
+#ifndef UC_HOIST_62
+#define UC_HOIST_62 3  // levels hoisted at <6, 2> (A/B: 0 / 2 / 3 / 4 -> 3509 / 3546 / 3568 / 3530 GLUPS)
+#endif
+// levels whose neighbours are shuffled before the ring wait (the rest after it)
 template <int T, int G>
-constexpr bool kHoistNeighbours = UC_HOIST_ALL == 1 || (UC_HOIST_ALL == 0 && !(T == 6 && G == 2));
+constexpr int kHoistLevels = UC_HOIST_ALL == 1 ? T : UC_HOIST_ALL == -1 ? 0 : (T == 6 && G == 2) ? UC_HOIST_62 : T;
 
 // One row of the T-level march: fetch the next A_k row, advance every level, store.
-template <int T, int NL, bool DIRI, bool STORE, bool HOIST>
+template <int T, int NL, bool DIRI, bool STORE, int HOIST>
 __device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
                                        const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
                                        float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
   float L[T], R[T];
-  if constexpr (HOIST) t_neighbours<T>(w1, L, R);  // overlaps the ring wait and the shared-memory load
+  t_neighbours<T, 0, HOIST>(w1, L, R);  // overlaps the ring wait and the shared-memory load
   const float4 nv = t_fetch(ring, full, empty, ST, NS, g, cur);
-  if constexpr (!HOIST) t_neighbours<T>(w1, L, R);
+  t_neighbours<T, HOIST, T>(w1, L, R);
   t_levels<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, L, R, out, pitch, acc);
 }
 
@@ -320,11 +325,11 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
   // the first 2T rows only fill the levels (rows >= 2T + 1 since a <= b)
 #pragma unroll
   for (int i = 0; i < 2 * T; ++i)
-    t_step<T, NL, DIRI, false, kHoistNeighbours<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
+    t_step<T, NL, DIRI, false, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
                                                       pitch, acc);
 #pragma unroll(kTUnroll)
   for (int i = 2 * T; i < rows; ++i)
-    t_step<T, NL, DIRI, true, kHoistNeighbours<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
+    t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
                                                      pitch, acc);
 }
 
