@@ -425,6 +425,7 @@ def run_ours(a):
                        "launch": launch_info},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches,
             "halo": halo, "pct_hbm_roofline": round(100 * glups / (world * peak / 8.0), 2),
+            "pct_hbm_roofline_note": "GLUPS vs the one-iteration-per-sweep roofline (8 B per point-iteration at the measured copy peak); above 100 because temporal blocking moves 8/T B per point-iteration; the kernel's own bandwidth fraction is roofline.frac",
         }
         print(json.dumps(line))
     if dist is not None:
