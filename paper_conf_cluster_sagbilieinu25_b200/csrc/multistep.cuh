@@ -280,35 +280,41 @@ __device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64
 }
 
 #ifndef UC_SKEW
-#define UC_SKEW 0  // A/B knob: 1 = skewed level schedule (t_levels_skew), 0 = the chained one
+#define UC_SKEW 0  // A/B knob: S > 0 = skewed level schedule in groups of S levels, 0 = fully chained
 #endif
+constexpr int kSkew = UC_SKEW > 0 ? UC_SKEW : 1;
 
-// Skewed schedule: level j+1 takes level j's row from the PREVIOUS step (pend[j-1]), so the T
-// level updates of one step are independent (T-way ILP instead of a T-deep chain) for T - 1 more
-// float4 registers.  Level j+1 emits row r - 2j - 1 at step i (r = a - T + i); the A_{k+T} row a
-// comes out at i = 3T - 1 and the march runs T - 1 drain steps past the last ring row.  Same
-// operations on the same operands as t_levels: bit-identical results.
+// Skewed schedule: the levels form groups of S = UC_SKEW; the first level of a group (j > 0,
+// j % S == 0) takes the previous group's row from the PREVIOUS step (pend[j-1]), so the groups of
+// one step are independent chains (T/S-way ILP) for D = (T-1)/S more float4 registers.  Level j+1
+// emits row r - j - 1 - j/S at step i (r = a - T + i); the A_{k+T} row a comes out at i = 2T + D
+// and the march runs D drain steps past the last ring row.  Same operations on the same operands
+// as t_levels: bit-identical results.
 template <int T, int NL, bool DIRI, bool STORE>
 __device__ __forceinline__ void t_levels_skew(float4 nv, const GhostLayout& g, int nx4, int a, int b, int i,
                                               float4 (&w0)[T], float4 (&w1)[T], float4 (&pend)[T],
                                               const float (&L)[T], const float (&R)[T], float*& out, size_t pitch,
                                               double& acc) {
-  float4 last = nv;
+  constexpr int S = kSkew;
+  float4 chain = nv, newp[T];
 #pragma unroll
-  for (int j = T - 1; j >= 0; --j) {
-    const float4 in = j == 0 ? nv : pend[j - 1];
-    const float4 o = row_update_lr<DIRI>(w0[j], w1[j], in, L[j], R[j], g.x4, nx4);  // level j+1, row r-2j-1
+  for (int j = 0; j < T; ++j) {
+    const float4 in = (j > 0 && j % S == 0) ? pend[j - 1] : chain;
+    const float4 o = row_update_lr<DIRI>(w0[j], w1[j], in, L[j], R[j], g.x4, nx4);  // level j+1
     if (NL == j + 1 && g.own) {
-      const int y = a - T + i - 2 * j - 1;
+      const int y = a - T + i - j - 1 - j / S;
       if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
     }
     w0[j] = w1[j];
     w1[j] = in;
-    if (j == T - 1) last = o;
-    else pend[j] = o;
+    if (j + 1 < T && (j + 1) % S == 0) newp[j] = o;
+    chain = o;
   }
+#pragma unroll
+  for (int j = 0; j + 1 < T; ++j)
+    if ((j + 1) % S == 0) pend[j] = newp[j];
   if (STORE) {
-    if (g.own) st4(out, last);
+    if (g.own) st4(out, chain);
     out += pitch;
   }
 }
@@ -369,8 +375,9 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
   RingCursor cur{0, 0u};
   float* out = dst + (size_t)a * pitch + 4 * (size_t)g.x4;  // the A_{k+T} row a comes out at i = 2T
 #if UC_SKEW
-  if constexpr (T > 1) {
-    constexpr int FILL = 3 * T - 1;  // steps before the first A_{k+T} row (a) comes out
+  if constexpr (T > 1 && (T - 1) / kSkew > 0) {
+    constexpr int D = (T - 1) / kSkew;  // skew delays along the level chain
+    constexpr int FILL = 2 * T + D;      // steps before the first A_{k+T} row (a) comes out
     constexpr int H = kHoistLevels<T, G>;
     float4 pend[T];
 #pragma unroll
@@ -388,7 +395,7 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
     for (int i = FILL; i < rows; ++i)
       t_step_skew<T, NL, DIRI, true, true, H>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, pend, out,
                                               pitch, acc);
-    for (int i = max(rows, FILL); i < rows + T - 1; ++i)  // drain: no ring row left
+    for (int i = max(rows, FILL); i < rows + D; ++i)  // drain: no ring row left
       t_step_skew<T, NL, DIRI, true, false, H>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, pend, out,
                                                pitch, acc);
     return;
