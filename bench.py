@@ -62,10 +62,10 @@ def parse():
                          "ranks time-slice the GPU, so the numbers are not a benchmark)")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
     ap.add_argument("--halo-only", action="store_true", help="skip e2e / cpu_baseline, keep the halo leg")
-    ap.add_argument("--cpu-sample-iters", type=int, default=3)
+    ap.add_argument("--cpu-sample-iters", type=int, default=12)
     ap.add_argument("--variant", type=int, default=-1,
                     help="0 register march, 1 TMA-staged, 2 dynamic tiles, 3 persistent, 4 two iterations per "
-                         "launch, 5 T iterations per launch (T = --tile-rows; -1: library default = 5, T = 4)")
+                         "launch, 5 T iterations per launch (T = --tile-rows; -1: library default = 5, T = 6)")
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--block-x", type=int, default=0)
@@ -238,6 +238,7 @@ def run_ours(a):
     for _ in range(a.warmup):
         step()
     coord.sync()
+    counts0 = J.launch_counts()
 
     # ---------------- timed region: K steps, events on the coordinator's stream
     barrier(dist)
@@ -253,80 +254,91 @@ def run_ours(a):
     clocks.mark_stop()
     barrier(dist)
     clk = clocks.stop()
+    counts1 = J.launch_counts()
     t_ms = e0.elapsed_time(e1)
     t_max = allreduce_max(dist, t_ms)
     ms_per_step = t_max / a.steps
     total_pts = pts_rank * world * ips * a.steps
     glups = total_pts / (t_max / 1e3) / 1e9
-    # iterations per launch: variant 4 = 2, variant 5 = T (device mode, n >= 2T, norm_every 0 or
-    # >= T), else 1; the last launch of a step may be shorter
+    # ---------------- the launches a step really runs (uc_jacobi_launch_plan; device counters agree)
     v = launch_info["variant"]
-    per_launch = 1
-    if a.mode == "device" and v == 4 and n >= 2 and a.norm_every != 1:
-        per_launch = 2
-    elif a.mode == "device" and v == 5:
-        per_launch = launch_info["tile_rows"]
-        while per_launch > 1 and not (n >= 2 * per_launch and (a.norm_every <= 0 or a.norm_every >= per_launch)):
-            per_launch -= 1
-    two = per_launch > 1
-    launches_per_step = -(-ips // per_launch)
-    launches = a.steps * launches_per_step + (
-        a.steps * ((ips + a.norm_every - 1) // a.norm_every) if a.mode == "host" else 0)
+    levels = launch_info["tile_rows"] if v == 5 else 1
+    plan = U.launch_plan(v, levels, mode, n, ips, a.norm_every)
+    per_launch = max(plan)
+    # our kernels in the timed region, from the device launch counters (host mode adds one
+    # norm_finish kernel per norm round; NCCL's own kernels are not counted)
+    ran = [c1 - c0 for c0, c1 in zip(counts0, counts1)]
+    assert ran[:len(ran)] == [sum(1 for t in plan if t == d) * a.steps for d in range(len(ran))], (ran, plan)
+    launches = sum(ran) + (a.steps * len(range(0, ips, a.norm_every)) if a.mode == "host" and a.norm_every > 0 else 0)
+    # which launches of a step carry the norm round (steps start at k = 0 mod ips)
+    norm_launch = []
+    kk = 0
+    for t in plan:
+        norm_launch.append(a.norm_every > 0 and any((kk + j) % a.norm_every == 0 for j in range(t)))
+        kk += t
+    ghosts = 2 if v == 5 and levels > 4 else 1
+    kname = (f"jacobi_t_kernel<{per_launch}, {ghosts}>" if v == 5 else
+             {4: "jacobi_two_step_kernel"}.get(v, "jacobi_iter_kernel"))
 
-    # ---------------- dominant kernel: per-launch events around single launches (no norm / norm)
-    def kernel_ms(compute_norm, reps, iters_per_launch):
-        es = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
-        buf = np.zeros(2, np.float64)
-        for s, e in es:
-            s.record(stream)
-            if iters_per_launch > 1:  # one multi-iteration launch (norm_every = T: one norm round in it)
-                J.run(coord, iters_per_launch, iters_per_launch if compute_norm else 0, False,
-                      norms_out=buf if compute_norm else None)
-            else:
-                J.step(coord, compute_norm, buf if compute_norm else None)
-            e.record(stream)
+    # ---------------- dominant kernel timed INSIDE a graph replay: a cached graph of L launches of
+    # depth per_launch (norm_every 0 / norm_every = depth: every launch with its norm round),
+    # replayed R times between CUDA events on the launching stream
+    def graph_kernel_ms(depth, with_norm, L=16, R=5):
+        iters = depth * L
+        ne = depth if with_norm else 0
+        buf = np.zeros(max(1, L), np.float64)
+        assert U.launch_plan(v, levels, mode, n, iters, ne) == [depth] * L
+        for _ in range(2):
+            J.run(coord, iters, ne, True, norms_out=buf if with_norm else None)
         coord.sync()
-        return statistics.mean(s.elapsed_time(e) for s, e in es)
+        barrier(dist)
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record(stream)
+        for _ in range(R):
+            J.run(coord, iters, ne, True, norms_out=buf if with_norm else None)
+        g1.record(stream)
+        coord.sync()
+        return g0.elapsed_time(g1) / (R * L)
 
-    barrier(dist)
-    k_plain = allreduce_max(dist, kernel_ms(False, 50, per_launch))
-    k_norm = allreduce_max(dist, kernel_ms(True, 10, per_launch))
-    # the timed steps have 1 norm round per norm_every iterations
-    nn = max(1, a.norm_every) if a.norm_every > 0 else ips
-    nn_launches = max(1, nn // per_launch)
-    k_avg = (k_plain * (nn_launches - 1) + k_norm) / nn_launches
+    k_plain = allreduce_max(dist, graph_kernel_ms(per_launch, False))
+    k_norm = allreduce_max(dist, graph_kernel_ms(per_launch, True))
+    n_dom = sum(1 for t in plan if t == per_launch)
+    n_dom_norm = sum(1 for t, nl in zip(plan, norm_launch) if t == per_launch and nl)
+    dom_ms = k_plain * (n_dom - n_dom_norm) + k_norm * n_dom_norm
     peak, peak_src = measured_peaks()
-    # algorithmic bytes per launch: every point of A_k read once, every point of the launch's
-    # last iterate written once -- 8 B per point per launch, for 1 or 2 iterations
+    # algorithmic bytes per launch: every point of A_k read once, every point of A_{k+T} written
+    # once -- 8 B per point per launch = 8/T B per point-iteration
     alg_bytes = 8.0 * pts_rank
     achieved = alg_bytes / (k_plain / 1e3) / 1e9
-    # variant 5 ghost layout: G = 2 ghost lanes per warp side when T > 4 (28 of 32 lanes owned)
-    ghosts = 2 if v == 5 and launch_info["tile_rows"] > 4 else 1
-    kname = {4: "jacobi_two_step_kernel", 5: f"jacobi_t_kernel<{per_launch}, {ghosts}>"}.get(v, "jacobi_iter_kernel") \
-        if two else (f"jacobi_t_kernel<1, {ghosts}>" if v == 5 else "jacobi_iter_kernel")
-    roof = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
+    sms = torch.cuda.get_device_properties(local).multi_processor_count
+    alu_peak = sms * 128 * sm_max_mhz() * 1e6 / 1e12
+    # FP32 work: 4 operations per point-iteration (3 FADD + 1 FMUL, never fused), T per launch,
+    # ghost lanes compute too (x 32 / (32 - 2G) for variant 5)
+    ops = 4.0 * pts_rank * per_launch * (32.0 / (32 - 2 * ghosts) if v == 5 else 1.0)
+    alu = ops / (k_plain / 1e3) / 1e12
+    # the two roofs as GLUPS ceilings at this depth: HBM moves 8/T B per point-iteration; the
+    # FP32 pipe does 4 (x ghost share) operations per point-iteration.  bound = the tighter one.
+    hbm_glups = peak / (8.0 / per_launch)
+    alu_glups = alu_peak * 1e3 / (ops / (pts_rank * per_launch))
+    tighter = "hbm" if hbm_glups <= alu_glups else "alu"
+    roof = {"bound": tighter, "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
             "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": ncu_traffic(nx, n, kname),
             "alg_bytes_per_launch": alg_bytes, "iterations_per_launch": per_launch,
             "hbm_bytes_per_point_iteration": 8.0 / per_launch,
+            "roof_glups": {"hbm": round(hbm_glups * world, 1), "alu": round(alu_glups * world, 1),
+                           "note": "ceilings at this launch depth (all ranks): HBM = peak / (8/T B per "
+                                   "point-iteration); ALU = FP32 peak / FP32 operations per point-iteration"},
             "kernel_ms": round(k_plain, 5), "kernel_norm_ms": round(k_norm, 5),
-            "kernel_share_of_step": round(k_avg * launches_per_step / ms_per_step, 4), "peak_source": peak_src}
-    # the FP32-pipe roof beside it: 4 FP32 operations per point-iteration (3 FADD +
-    # 1 FMUL, never fused), T iterations per launch, ghost lanes compute too (x 32 / (32 - 2G));
-    # peak = SMs x 128 FP32 lanes x max SM clock
-    sms = torch.cuda.get_device_properties(local).multi_processor_count
-    alu_peak = sms * 128 * sm_max_mhz() * 1e6 / 1e12
-    ops = 4.0 * pts_rank * per_launch * (32.0 / (32 - 2 * ghosts) if v == 5 else 1.0)
-    alu = ops / (k_plain / 1e3) / 1e12
+            "kernel_timing": "inside a CUDA-graph replay of 16 launches (events on the launching stream)",
+            "launch_plan_per_step": plan,
+            "kernel_share_of_step": round(dom_ms / ms_per_step, 4), "peak_source": peak_src}
+    if tighter == "alu":  # report the FP32 roof as the primary figure
+        roof.update({"achieved": round(alu, 3), "peak": round(alu_peak, 2), "unit": "TFLOP/s",
+                     "frac": round(alu / alu_peak, 4)})
     roof["alu"] = {"bound": "alu", "achieved": round(alu, 3), "peak": round(alu_peak, 2), "unit": "TFLOP/s",
                    "frac": round(alu / alu_peak, 4), "flops_per_launch": ops,
-                   "peak_source": f"{sms} SMs x 128 FP32 lanes x {sm_max_mhz():.0f} MHz"}
-    if two:
-        # the one-iteration kernel in the same geometry, for comparison (8 B per point per iteration)
-        k1 = allreduce_max(dist, kernel_ms(False, 30, 1))
-        roof["one_iteration_kernel"] = {"kernel": f"jacobi_t_kernel<1, {ghosts}>" if v == 5 else "jacobi_iter_kernel",
-                                        "kernel_ms": round(k1, 5),
-                                        "achieved": round(alg_bytes / (k1 / 1e3) / 1e9, 1),
-                                        "glups": round(pts_rank * world / (k1 / 1e3) / 1e9, 1)}
+                   "peak_source": f"{sms} SMs x 128 FP32 lanes x {sm_max_mhz():.0f} MHz (derived, DESIGN.md §5)"}
+    roof["hbm"] = {"achieved": round(achieved, 1), "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4)}
 
     # ---------------- halo exchange overlap (differential, §8 d): same slab, no neighbours
     halo = None
@@ -389,7 +401,7 @@ def run_ours(a):
             times[pipelined] = allreduce_max(dist, max(f0.elapsed_time(f1), f0.elapsed_time(f2)))
         te, ts = times[True], times[False]
         e2e = {"value": round(pts_rank * world * ips * ke / (te / 1e3) / 1e9, 3), "unit": UNIT,
-               "h2d_bytes_per_step": slab_elems * 4, "d2h_bytes_per_step": slab_elems * 4 + 8 * max(1, ips // nn),
+               "h2d_bytes_per_step": slab_elems * 4, "d2h_bytes_per_step": slab_elems * 4 + 8 * (len(range(0, ips, a.norm_every)) if a.norm_every > 0 else 0),
                "steps": ke, "ms_per_step": round(te / ke, 3),
                "pipeline": "2 solvers on 2 streams alternate steps (H2D of step i+1 overlaps compute + D2H of step i)",
                "serial_value": round(pts_rank * world * ips * ke / (ts / 1e3) / 1e9, 3),
@@ -405,9 +417,10 @@ def run_ours(a):
     env.finalize()
 
     # ---------------- oracle on the host cores (rank 0, N = 1)
-    cpu = None
+    cpu = cpu_par = None
     if rank == 0 and world == 1 and not a.no_extras and not a.halo_only:
-        cpu = cpu_baseline(nx, a.ny_per_gpu, a.cpu_sample_iters)
+        cpu = cpu_baseline(nx, a.ny_per_gpu, a.cpu_sample_iters, a.norm_every)
+        cpu_par = cpu_parallel(nx, a.ny_per_gpu, 10, a.norm_every)
 
     if rank == 0:
         line = {
@@ -423,7 +436,8 @@ def run_ours(a):
                        "parallelism": f"y-slab x{world}", "l2": "inputs > L2 (2 slabs x "
                        f"{(n + 2) * nx * 4 / 2**20:.0f} MiB per GPU vs 126 MB L2), no flush",
                        "launch": launch_info},
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk, "gpu_launches": launches,
+            "roofline": roof, "cpu_baseline": cpu, "cpu_parallel": cpu_par, "e2e": e2e, "clocks": clk, "gpu_launches": launches,
+            "gpu_launches_by_depth": {str(d): c for d, c in enumerate(ran) if c},
             "halo": halo, "pct_hbm_roofline": round(100 * glups / (world * peak / 8.0), 2),
             "pct_hbm_roofline_note": "GLUPS vs the one-iteration-per-sweep roofline (8 B per point-iteration at the measured copy peak); above 100 because temporal blocking moves 8/T B per point-iteration; the kernel's own bandwidth fraction is roofline.frac",
         }
@@ -517,57 +531,95 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
                     f"rows + waits, x{per_launch} rounds"}
 
 
-def cpu_baseline(nx, ny, iters):
-    """The oracle as it stands (single-threaded C, -O2), on a bounded sample of the workload."""
+def cpu_baseline(nx, ny, iters, norm_every):
+    """The oracle as it stands (single-threaded C, -O2) on a bounded sample of the workload: one
+    oracle_jacobi_run of `iters` iterations of the full rank-0 grid (the norm every norm_every
+    iterations, as in the timed steps), timed around the C call only."""
     import oracle
     from inputs import gen
     oracle.build()
     g = gen.global_field(nx, ny, "ring")
     t = time.perf_counter()
-    oracle.jacobi_run(g, iters, "ring", 1)
+    oracle.jacobi_run(g, iters, "ring", norm_every)
     dt = time.perf_counter() - t
     return {"value": round(ny * (nx - 2) * iters / dt / 1e9, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{iters} iterations (norm every iteration) of the full {nx}x{ny} ring grid, "
-                      f"{dt:.1f} s, host {os.cpu_count()} cores visible, 1 used"}
+            "sample": f"one oracle run of {iters} iterations (norm every {norm_every}) of the full {nx}x{ny} ring "
+                      f"grid, {dt:.1f} s incl. the wrapper's copy of the 1 GiB array; host {os.cpu_count()} "
+                      "cores visible, 1 used (the oracle is single-threaded by design)"}
+
+
+def cpu_parallel(nx, ny, iters, norm_every):
+    """The same loop on every host core (benchmarks/cpu_omp, OpenMP C, bit-identical grid --
+    tests/test_cpu_omp.py): the multi-core host baseline beside the single-core oracle."""
+    import numpy as np
+
+    from benchmarks import cpu_omp
+    from inputs import gen
+    cpu_omp.build()
+    g = np.ascontiguousarray(gen.global_field(nx, ny, "ring"), dtype=np.float32)
+    cpu_omp.jacobi_run(g, 1, "ring", 0, inplace=True)  # page in, spin up the thread pool
+    t = time.perf_counter()
+    cpu_omp.jacobi_run(g, iters, "ring", norm_every, inplace=True)
+    dt = time.perf_counter() - t
+    return {"value": round(ny * (nx - 2) * iters / dt / 1e9, 4), "unit": UNIT, "cores": cpu_omp.threads(),
+            "kind": "openmp (same loop as the oracle, bit-identical grid)",
+            "sample": f"{iters} iterations (norm every {norm_every}) of the full {nx}x{ny} ring grid, {dt:.2f} s"}
 
 
 # ----------------------------------------------------------------------------- reference arm
 def run_reference(a):
     """The oracle (plain single-threaded C over the global grid) on the host cores, as the
-    reference arm: each step is a bounded sample (a.cpu_sample_iters... one iteration) of the
-    same 16384 x 16384-per-GPU workload."""
+    reference arm: rank 0 only.  The warm-up is one oracle run of W iterations, the timed region
+    ONE oracle run of K iterations (each "step" = one iteration of the 16384^2 rank-0 grid with
+    the step's norm cadence), so the wrapper's array copies are paid once, not per step."""
     rank, world, _ = dist_env()
     if rank != 0:
         return
+    import numpy as np
+
     import oracle
     from inputs import gen
     oracle.build()
     nx, ny = a.nx, a.ny_per_gpu
     g = gen.global_field(nx, ny, "ring")
-    iters = 1
-    for _ in range(a.warmup):
-        g, _s = oracle.jacobi_run(g, iters, "ring", 1)
+    g, _s = oracle.jacobi_run(g, a.warmup, "ring", a.norm_every)
     t = time.perf_counter()
-    for _ in range(a.steps):
-        g, _s = oracle.jacobi_run(g, iters, "ring", 1)
+    g, _s = oracle.jacobi_run(g, a.steps, "ring", a.norm_every)
     dt = time.perf_counter() - t
-    v = ny * (nx - 2) * iters * a.steps / dt / 1e9
+    assert np.isfinite(g[1, 1])
+    v = ny * (nx - 2) * a.steps / dt / 1e9
     line = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(dt / a.steps * 1e3, 2),
             "higher_is_better": True, "scaling": a.scaling, "vs_baseline": None, "dtype": "f32",
             "data": "synthetic",
             "config": {"workload": f"jacobi2d_{nx}x{ny}_per_gpu_{a.mode}_ring", "nx": nx, "ny_global": ny,
-                       "sample": "1 iteration per step (norm each iteration) of the rank-0 grid"},
+                       "sample": f"1 iteration per step of the rank-0 {nx}x{ny} grid (norm every {a.norm_every}); "
+                                 "K steps timed as one oracle run"},
             "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"{a.steps} steps x 1 iteration of {nx}x{ny}"},
+                             "sample": f"one oracle run of {a.steps} iterations of {nx}x{ny}, {dt:.1f} s"},
             "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
+
+
+def spawn_ranks(a):
+    """`bench.py --gpus N` without a torchrun environment: launch N ranks (one per GPU) with
+    torch.distributed.run on 127.0.0.1 and relay their output (rank 0 prints the JSON line)."""
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd, cwd=ROOT)
 
 
 def main():
     a = parse()
     if a.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(a))
     if a.impl == "reference":
         run_reference(a)
     else:

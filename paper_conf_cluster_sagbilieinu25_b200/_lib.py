@@ -78,6 +78,7 @@ _SIGS = {
     "uc_jacobi_step": (i32, [vp, vp, i32, vp]),
     "uc_jacobi_run": (i32, [vp, vp, i32, i32, vp, i32]),
     "uc_jacobi_num_norms": (i32, [vp, i32, i32]),
+    "uc_jacobi_launch_counts": (i32, [vp, P(u64), i32]),
     "uc_jacobi_launch_plan": (i32, [i32, i32, i32, i32, i32, i32, P(i32), i32]),
     "uc_jacobi_copy_in": (i32, [vp, vp]),
     "uc_jacobi_copy_out": (i32, [vp, vp, vp, i32]),

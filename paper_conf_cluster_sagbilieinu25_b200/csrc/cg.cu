@@ -5,7 +5,7 @@
 // the paper gathers it with AllGatherv -- and two dot products reduced over all ranks
 // (P:430).  Three kernels per iteration, all scalars on the device (no host round trip, so a
 // CUDA graph of many iterations replays exactly):
-//   K1 cg_spmv:     q = A p (sub-warp of 8 lanes per CSR row) fused with the partial p.q; the
+//   K1 cg_spmv:     q = A p (sub-warp of 4 lanes per CSR row by default, uc_cg_set_launch) fused with the partial p.q; the
 //                   last block (ticket) reduces the block partials in order and, in device mode,
 //                   runs the one-shot cross-rank allreduce and sets alpha = rr / p.q.
 //   K2 cg_update:   x += alpha p, r -= alpha q fused with the partial r.r; the last block
@@ -306,7 +306,7 @@ struct uc_cg {
   long long k = 0;
   int mode = -1;  // launch mode that drives this solver (fixed after the first run)
   cudaStream_t aux = nullptr;
-  std::vector<JacobiGraph> graphs;  // (iters, mode, stream) -> exec
+  GraphCache graphs;  // (iters, mode, stream, coordinator, timeout) -> exec
 };
 
 namespace {
@@ -398,7 +398,6 @@ int cg_configure(uc_cg* cg, int tpr, int unroll) {
   cg->unroll = unroll;
   cg->spmv_grid = sg;
   cg->grid = vg;
-  for (auto& g : cg->graphs) cudaGraphExecDestroy(g.exec);
   cg->graphs.clear();
   return UC_OK;
 }
@@ -535,8 +534,10 @@ int uc_cg_run(uc_coord* k, uc_cg* cg, int iters, double* rr_out, int use_graph) 
   if (k->mode != UC_MODE_DEVICE) UC_TRY(ensure_nccl(k));
   if (use_graph && k->stream) {
     JacobiGraph* g = nullptr;
-    for (auto& x : cg->graphs)
-      if (x.iters == iters && x.mode == (int)k->mode && x.stream == k->stream) g = &x;
+    for (auto& x : cg->graphs.graphs)
+      if (x.iters == iters && x.mode == (int)k->mode && x.stream == k->stream && x.coord == k &&
+          x.timeout_ns == k->timeout_ns)
+        g = &x;
     if (!g) {
       UC_CUDA(cudaStreamBeginCapture(k->stream, cudaStreamCaptureModeThreadLocal));
       int rc = UC_OK;
@@ -552,13 +553,15 @@ int uc_cg_run(uc_coord* k, uc_cg* cg, int iters, double* rr_out, int use_graph) 
       ng.iters = iters;
       ng.mode = (int)k->mode;
       ng.stream = k->stream;
+      ng.coord = k;
+      ng.timeout_ns = k->timeout_ns;
       e = cudaGraphInstantiate(&ng.exec, graph, 0);
       cudaGraphDestroy(graph);
       if (e == cudaSuccess) e = cudaGraphUpload(ng.exec, k->stream);
       if (e == cudaSuccess) e = cudaStreamSynchronize(k->stream);
       if (e != cudaSuccess) return fail(UC_ERR_CUDA, "graph build: %s", cudaGetErrorString(e));
-      cg->graphs.push_back(ng);
-      g = &cg->graphs.back();
+      cg->graphs.add(k, ng);
+      g = &cg->graphs.graphs.back();
       UC_TRY(uc_comm_barrier(cg->comm, k->stream));  // building a graph is collective (see Jacobi)
     }
     UC_CUDA(cudaGraphLaunch(g->exec, k->stream));
@@ -610,7 +613,7 @@ int uc_cg_destroy(uc_cg* cg) {
   uc_comm* c = cg->comm;
   UC_CUDA(cudaSetDevice(c->env->device));
   UC_CUDA(cudaStreamSynchronize(cg->aux));
-  for (auto& g : cg->graphs) cudaGraphExecDestroy(g.exec);
+  cg->graphs.release();
   UC_TRY(uc_mem_free_symmetric(cg->pfull));
   UC_TRY(uc_mem_free_symmetric(cg->ctrl));
   cudaFree(cg->rowptr);

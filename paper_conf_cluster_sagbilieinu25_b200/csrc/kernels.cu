@@ -541,6 +541,7 @@ __global__ void __launch_bounds__(kMaxBlock + 32, 4) jacobi_persistent_kernel(co
     if (s_last) {
       __threadfence();
       p.k_dev[0] = k0 + (uint64_t)iters;
+      p.launch_hist[0] += 1ull;  // persistent launches are counted in slot 0
       *p.done = 0;
       __threadfence();
     }

@@ -28,6 +28,8 @@ int fail(int status, const char* fmt, ...) {
   return status;
 }
 
+static void flush_pending(uc_coord* k);
+
 int enqueue_d2h_f64(uc_coord* k, double* host, const double* dev, double* stage, size_t n) {
   if (!host || n == 0) return UC_OK;
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
@@ -39,6 +41,14 @@ int enqueue_d2h_f64(uc_coord* k, double* host, const double* dev, double* stage,
     UC_CUDA(cudaMemcpyAsync(host, dev, n * sizeof(double), cudaMemcpyDeviceToHost, k->stream));
     return UC_OK;
   }
+  // a stage slot still pending (more than the history's worth of outputs enqueued since the
+  // last uc_coord_sync) is completed first, so the earlier output never receives a later value
+  for (const auto& c : k->pending)
+    if (c.src < stage + n && stage < c.src + c.n) {
+      UC_CUDA(cudaStreamSynchronize(k->stream));
+      flush_pending(k);
+      break;
+    }
   UC_CUDA(cudaMemcpyAsync(stage, dev, n * sizeof(double), cudaMemcpyDeviceToHost, k->stream));
   k->pending.push_back({host, stage, n});
   return UC_OK;
@@ -64,6 +74,39 @@ static uint64_t host_hash() {
 }  // namespace uc
 
 using namespace uc;
+
+void GraphCache::add(uc_coord* k, const JacobiGraph& g) {
+  graphs.push_back(g);
+  if (std::find(coords.begin(), coords.end(), k) == coords.end()) {
+    coords.push_back(k);
+    k->caches.push_back(this);
+  }
+}
+
+void GraphCache::clear() {
+  for (auto& g : graphs) cudaGraphExecDestroy(g.exec);
+  graphs.clear();
+}
+
+void GraphCache::forget(uc_coord* k) {
+  for (auto it = graphs.begin(); it != graphs.end();) {
+    if (it->coord == k) {
+      cudaGraphExecDestroy(it->exec);
+      it = graphs.erase(it);
+    } else {
+      ++it;
+    }
+  }
+  coords.erase(std::remove(coords.begin(), coords.end(), k), coords.end());
+  k->caches.erase(std::remove(k->caches.begin(), k->caches.end(), this), k->caches.end());
+}
+
+void GraphCache::release() {
+  clear();
+  for (uc_coord* k : coords) k->caches.erase(std::remove(k->caches.begin(), k->caches.end(), this), k->caches.end());
+  coords.clear();
+}
+
 
 int uc_env::allgather(const void* send, void* recv, size_t bytes) {
   if (size == 1) {
@@ -428,9 +471,11 @@ int uc_coord_create(uc_comm* c, uc_mode mode, void* stream, uc_coord** out) {
 
 int uc_coord_destroy(uc_coord* k) {
   if (!k) return fail(UC_ERR_ARG, "coord is NULL");
-  if (k->live_jacobi_users) return fail(UC_ERR_STATE, "coordinator still in use");
   UC_CUDA(cudaSetDevice(k->comm->env->device));
   if (cudaStreamSynchronize(k->stream) == cudaSuccess) flush_pending(k);
+  // solvers' graphs captured on this coordinator point at its error word / NCCL communicator:
+  // they go with it (a later coordinator never replays them)
+  while (!k->caches.empty()) k->caches.back()->forget(k);
   if (k->nccl) ncclCommDestroy(k->nccl);
   if (k->ar_scratch) UC_TRY(uc_mem_free_symmetric(k->ar_scratch));
   if (k->coll_flags) UC_TRY(uc_mem_free_symmetric(k->coll_flags));

@@ -196,6 +196,7 @@ __device__ inline void finish_iteration(const JacobiParams& p, bool do_norm, dou
     if (do_norm) norm_publish(p, tot);
     p.k_dev[0] = p.k_dev[0] + (unsigned long long)advance;
     if ((advance & 1) == 0) p.k_dev[2] = p.k_dev[2] ^ 1ull;  // A_{k+advance} went to the other slab
+    p.launch_hist[advance < 15 ? advance : 15] += 1ull;      // what really ran (uc_jacobi_launch_counts)
     *p.done = 0;
     *p.work = 0;  // variant 2 tile counter
     __threadfence();

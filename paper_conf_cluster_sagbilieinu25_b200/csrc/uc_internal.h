@@ -61,6 +61,7 @@ struct JacobiParams {
   double* norm_slot[UC_MAX_RANKS];     // rank q's norm slots: [2][P] doubles
   uint64_t* norm_flag[UC_MAX_RANKS];   // rank q's norm flags: [2][P] u64 (stride kFlagStride)
   unsigned long long* k_dev;           // local [k, norm round m, slab parity offset, -]
+  unsigned long long* launch_hist;     // local [16]: completed launches by iterations per launch
   unsigned int* done;                  // local block ticket
   unsigned int* work;                  // local dynamic tile counter (variant 2)
   unsigned int* nbar;                  // local [count, generation] norm grid barrier (variant 3)
@@ -204,6 +205,8 @@ struct uc_mem {
   std::vector<bool> ipc_opened; // per rank: close with cudaIpcCloseMemHandle
 };
 
+struct GraphCache;
+
 struct uc_coord {
   uc_comm* comm = nullptr;
   uc_mode mode = UC_MODE_HOST;
@@ -221,19 +224,34 @@ struct uc_coord {
   float* nccl_scratch = nullptr;       // host-mode barrier operand
   uint64_t p2p_epoch[3][UC_MAX_RANKS] = {};  // signal base of the next uc_p2p_bench call, per (pattern, peer)
   unsigned int* p2p_bar = nullptr;     // grid barrier [count, gen] of the p2p kernel
-  int live_jacobi_users = 0;
   struct PendingCopy {
     double* dst;
     const double* src;
     size_t n;
   };
   std::vector<PendingCopy> pending;    // staged pageable outputs, copied at uc_coord_sync
+  std::vector<GraphCache*> caches;     // solvers' graph caches holding graphs built on this coordinator
 };
 
+// A captured run.  The graph bakes in its coordinator's stream, error word, spin timeout and (host /
+// partial mode) NCCL communicator, so the coordinator and its timeout are part of the key and a
+// coordinator's graphs die with it (GraphCache::forget from uc_coord_destroy).
 struct JacobiGraph {
   int iters = 0, norm_every = 0, parity = 0, flip = 0, mode = -1;
   cudaStream_t stream = nullptr;
+  const uc_coord* coord = nullptr;
+  unsigned long long timeout_ns = 0;
   cudaGraphExec_t exec = nullptr;
+};
+
+// The graphs one solver (Jacobi or CG) built, and the coordinators that know about this cache.
+struct GraphCache {
+  std::vector<JacobiGraph> graphs;
+  std::vector<uc_coord*> coords;
+  void add(uc_coord* k, const JacobiGraph& g);  // registers the cache with k
+  void clear();                                 // destroy every graph (geometry change)
+  void forget(uc_coord* k);                     // destroy k's graphs and unregister (k is being destroyed)
+  void release();                               // solver destroyed: clear + unregister
 };
 
 struct uc_jacobi {
@@ -255,6 +273,7 @@ struct uc_jacobi {
   int max_strips = 0;           // flag capacity per side = ceil(nx/4 / 32)
   // local device state
   unsigned long long* k_dev = nullptr;
+  unsigned long long* launch_hist = nullptr;  // [16] completed launches by iterations per launch
   unsigned int* done = nullptr;
   double* partials = nullptr;
   uint64_t* blk_done = nullptr;  // [partials_cap] per-block completed iteration (variant 3)
@@ -267,5 +286,5 @@ struct uc_jacobi {
   int last_mode = -1;            // mode of the coordinator that ran the previous iterations
   int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
   int partials_cap = 0;
-  std::vector<JacobiGraph> graphs;
+  GraphCache graphs;
 };

@@ -18,7 +18,7 @@ from typing import Callable, Optional
 
 import numpy as np
 
-from ._lib import (ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
+from ._lib import (UC_OK, UC_ERR_TIMEOUT, UC_ERR_STATE, UC_ERR_ARG, ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
                    UC_MAX, UC_MIN, UC_P2P_HALO, UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_PROD, UC_SUM, UC_TOPO_CHAIN,
                    UC_TOPO_NONE, UC_TOPO_RING, UC_U64,
                    UCError, check, lib)
@@ -344,6 +344,13 @@ class Jacobi:
         """COLLECTIVE (see uc_jacobi_set_launch)."""
         check(lib.uc_jacobi_set_launch(self.h, variant, block_x, blocks_per_sm, stages, tile_rows),
               "uc_jacobi_set_launch")
+
+    def launch_counts(self) -> list:
+        """uc_jacobi_launch_counts: completed launches by iterations per launch (index t = 1..8;
+        0 = persistent launches), from device counters -- what really ran.  After Coord.sync."""
+        buf = (C.c_uint64 * 16)()
+        check(lib.uc_jacobi_launch_counts(self.h, buf, 16), "uc_jacobi_launch_counts")
+        return list(buf)
 
     def launch_info(self) -> dict:
         v, g, b, s, c, st, tr = (C.c_int() for _ in range(7))

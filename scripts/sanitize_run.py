@@ -31,16 +31,30 @@ def main():
         dict(P=2, mode="device", variant=5, T=3, ne=3), dict(P=1, mode="device", variant=5, T=2, ne=2),
         dict(P=1, mode="host", variant=5, T=4), dict(P=1, mode="partial", variant=5, T=4),
     ]
+    # the shipped default, jacobi_t_kernel<6, 2> (two ghost lanes, five h-row levels), at P = 1
+    # (self-exchange), P = 2 (top == bottom) and P = 3 (distinct peers); ne = 6 keeps every launch
+    # at T = 6 (a norm cadence below T demotes launches)
+    t6 = [dict(P=1, mode="device", variant=5, T=6, ne=6, iters=13), dict(P=2, mode="device", variant=5, T=6, ne=0, iters=12),
+          dict(P=3, mode="device", variant=5, T=6, ne=6, iters=12)]
+    if os.environ.get("UC_SANITIZE_T6_ONLY"):
+        cases = t6
+    else:
+        cases += t6
     if len(sys.argv) > 1:
         cases = cases[: int(sys.argv[1])]
-    nx, ny, iters = 132, 24, 9
+    nx, ny = 132, 24
     for c in cases:
         P = c["P"]
+        iters = c.get("iters", 9)
         ne = c.get("ne", 2)
         res = solve_gpu(nx, ny * P, P, "ring", c["mode"], iters, ne if c["mode"] != "partial" or P == 1 else 0,
                         variant=c["variant"], tile_rows=c.get("T", 0), use_graph=False)
         want, _ = oracle.jacobi_run(gen.global_field(nx, ny * P, "ring"), iters, "ring")
         assert_slabs_equal_global(res["final"], want, P, "ring")
+        if c["variant"] == 5 and c.get("T", 0) == 6:
+            import paper_conf_cluster_sagbilieinu25_b200 as U
+            plan = U.launch_plan(5, 6, 1, ny, iters, ne)
+            assert plan[:2] == [6, 6], plan
         print("ok", c, flush=True)
     print("SANITIZE_RUN_DONE")
 

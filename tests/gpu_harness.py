@@ -58,7 +58,12 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
             coord.sync()
             final = J.copy_out(coord)
             info = J.launch_info()
-            return slab0, final, norms, info
+            counts = J.launch_counts()
+            want = expected_counts(U, info, MODES[mode], ny // P, iters, norm_every, stepwise, chunks_of_run)
+            if want is not None:  # the launches that really ran are the plan's (no silent demotion)
+                assert counts == want, (f"rank {rank}: launches by iterations per launch {counts[:9]} != "
+                                        f"plan {want[:9]} ({info})")
+            return slab0, final, norms, info, counts
         finally:
             comm.barrier()
             J.destroy()
@@ -68,7 +73,24 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
 
     res = run_ranks(P, body)
     return {"init": [r[0] for r in res], "final": [r[1] for r in res], "norms": res[0][2],
-            "norms_all": [r[2] for r in res], "launch": res[0][3]}
+            "norms_all": [r[2] for r in res], "launch": res[0][3], "counts": res[0][4],
+            "counts_all": [r[4] for r in res]}
+
+
+def expected_counts(U, info, mode, n_local, iters, norm_every, stepwise=False, chunks_of_run=None):
+    """Histogram (launches by iterations per launch) the launch plan predicts for a run, or None
+    where launches are not one-per-plan-entry (the persistent variant 3 in device mode)."""
+    v = info["variant"]
+    if v == 3 and mode == 1:
+        return None
+    h = [0] * 16
+    if stepwise:
+        h[1] = iters
+        return h
+    for it in (chunks_of_run or [iters]):
+        for t in U.launch_plan(v, info["tile_rows"] if v == 5 else 1, mode, n_local, it, norm_every):
+            h[t] += 1
+    return h
 
 
 def bits(a):

@@ -28,6 +28,8 @@ def main():
     ap.add_argument("--mode", default="device")
     ap.add_argument("--topology", default="ring")
     ap.add_argument("--same-device", action="store_true")
+    ap.add_argument("--variant", type=int, default=-1)
+    ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--out", required=True)
     a = ap.parse_args()
     rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
@@ -42,10 +44,13 @@ def main():
     coord = U.Coord(comm, mode, stream.cuda_stream)
     coord.set_timeout(20.0)
     J = U.Jacobi(comm, a.nx, a.ny)
+    if a.variant >= 0:
+        J.set_launch(a.variant, 0, 0, 0, a.tile_rows)
     norms = J.run(coord, a.iters, a.norm_every, use_graph=True)
     coord.sync()
     slab = J.copy_out(coord)
-    np.savez(os.path.join(a.out, f"rank{rank}.npz"), slab=slab, norms=norms)
+    counts = np.array(J.launch_counts(), np.uint64)
+    np.savez(os.path.join(a.out, f"rank{rank}.npz"), slab=slab, norms=norms, counts=counts)
     comm.barrier()
     J.destroy()
     coord.destroy()

@@ -27,12 +27,14 @@ def window_oracle(nx, ny, y0, y1, k, topology="ring"):
     return out[k + 1:k + 1 + (y1 - y0 + 1)]
 
 
-@pytest.mark.parametrize("variant", [5, 4, 1])
-def test_weak_scaling_8x16384sq_sampled_rows(variant):
+@pytest.mark.parametrize("variant,k,ne", [(5, 12, 6), (5, 4, 4), (4, 4, 4), (1, 4, 4)])
+def test_weak_scaling_8x16384sq_sampled_rows(variant, k, ne):
+    """variant 5 at k = 12, norm every 6: two launches of the shipped jacobi_t_kernel<6, 2> with 8
+    distinct ranks; k = 4: one T = 4 launch."""
     import torch
 
     import paper_conf_cluster_sagbilieinu25_b200 as U
-    P, nx, n, k = 8, 16384, 16384, 4
+    P, nx, n = 8, 16384, 16384
     ny = P * n
     edge = 6  # owned rows sampled at each end of a slab, plus both halo rows
 
@@ -47,13 +49,15 @@ def test_weak_scaling_8x16384sq_sampled_rows(variant):
             J.set_launch(variant)
         try:
             comm.barrier()
-            J.run(co, k, 4, use_graph=True)  # variant 5: one launch of T = 4 iterations
+            J.run(co, k, ne, use_graph=True)
+            co.sync()
+            counts = J.launch_counts()
             co.sync()
             top = J.copy_rows(co, 0, edge + 1)                  # halo row 0 + owned rows 1..edge
             bot = J.copy_rows(co, n + 1 - edge, edge + 1)       # owned rows n-edge+1..n + halo n+1
             mid = J.copy_rows(co, n // 2, 3)
             info = J.launch_info()
-            return top, bot, mid, info
+            return top, bot, mid, info, counts
         finally:
             comm.barrier()
             J.destroy()
@@ -63,8 +67,12 @@ def test_weak_scaling_8x16384sq_sampled_rows(variant):
 
     res = run_ranks(P, body)
     assert res[0][3]["variant"] == variant
+    if variant == 5:
+        for r in range(P):
+            c = res[r][4]
+            assert (c[6], sum(c)) == ((2, 2) if k == 12 else (0, 1)), c
     for r in range(P):
-        top, bot, mid, _ = res[r]
+        top, bot, mid, _, _ = res[r]
         g0 = r * n  # global computed row of slab row 1
         # slab row j <-> global computed row g0 + j - 1 (ring-wrapped for the halo rows)
         want_top = window_oracle(nx, ny, g0 - 1, g0 + edge - 1, k)

@@ -183,3 +183,98 @@ def test_config2_strong_16384_over_8_ranks():
 @pytest.mark.parametrize("T", [4, 8])
 def test_config1_4096_2ranks_1000_iterations(T):
     _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, **_v5(T))
+
+
+# ---------------------------------------------------------------------------------------------
+# The shipped default, jacobi_t_kernel<6, 2>, where the multi-rank protocol can break: distinct
+# top and bottom peers (P >= 3), the chain ends, full-size geometry.  A norm cadence below T
+# demotes launches, so these runs use norm_every 0 or a multiple of 6 and assert (through the
+# device launch counters, uc_jacobi_launch_counts) that T = 6 launches really ran.
+
+@pytest.mark.parametrize("P", [3, 4, 8])
+@pytest.mark.parametrize("topology,ne", [("ring", 0), ("ring", 6), ("dirichlet", 12)])
+def test_t6_distinct_peers(P, topology, ne):
+    res = _check(1028, 24 * P, P, topology, "device", 18, norm_every=ne)  # library default: T = 6
+    assert res["launch"]["variant"] == 5 and res["launch"]["tile_rows"] == 6
+    for c in res["counts_all"]:
+        assert c[6] == 3 and sum(c) == 3, c
+
+
+@pytest.mark.parametrize("P,rows", [(3, 12), (4, 13), (2, 12)])
+def test_t6_thinnest_slabs(P, rows):
+    """n = 2T = 12 (every chunk is a boundary chunk) and n = 13 (ragged), wide enough for two
+    strips per rank."""
+    for topology in ("ring", "dirichlet"):
+        res = _check(2052, rows * P, P, topology, "device", 12, norm_every=6)
+        assert all(c[6] == 2 for c in res["counts_all"]), res["counts_all"]
+
+
+def test_t6_random_values_p3():
+    nx, ny = 1028, 72
+    rng = np.random.default_rng(6)
+    init = rng.random((ny + 2, nx), dtype=np.float32)
+    init[0], init[-1] = init[ny], init[1]
+    res = _check(nx, ny, 3, "ring", "device", 24, norm_every=6, init=init)
+    assert res["counts"][6] == 4
+
+
+def test_t6_config1_default():
+    """configs[1] (4096^2, 2 ranks, 1000 iterations, norm every 100) at the library default:
+    166 launches of T = 6 and one of T = 4."""
+    res = _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100)
+    assert res["launch"]["tile_rows"] == 6
+    for c in res["counts_all"]:
+        assert c[6] == 166 and c[4] == 1 and sum(c) == 167, c
+
+
+def test_t6_config3_two_ranks():
+    """configs[3] at P = 2 (16384 x 32768 global, 16384^2 per rank: the bench's per-GPU geometry
+    with real neighbours), 13 iterations with a norm every 6: launches 6, 6, 1."""
+    res = _check(16384, 32768, 2, "ring", "device", 13, norm_every=6)
+    for c in res["counts_all"]:
+        assert c[6] == 2 and c[1] == 1, c
+
+
+def test_two_virtual_ranks_need_concurrent_kernels():
+    """States the requirement the virtual-rank tests rely on: two ranks on ONE GPU run their
+    device-mode kernels on two streams, and each kernel spins on flags the other sets, so both
+    grids must make progress at the same time.  CUDA does not guarantee concurrent kernels (a
+    profiler or MPS serialises them -- the paper notes the missing preemptive scheduling,
+    P:115), which is why smoke() runs P = 1.  When the peer's kernel does NOT run alongside
+    (here: rank 1 launches only after rank 0's spin timeout), the waits are bounded and both
+    ranks report UC_ERR_TIMEOUT instead of hanging the device."""
+    import time
+
+    import torch
+
+    import paper_conf_cluster_sagbilieinu25_b200 as U
+    from vranks import run_ranks
+
+    def body(rank, P, ag):
+        env = U.Env(rank, P, 0, ag)
+        comm = U.Comm(env, *U.ring_neighbours(rank, P))
+        st = torch.cuda.Stream()
+        co = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
+        co.set_timeout(0.5)
+        J = U.Jacobi(comm, 1028, 48)
+        comm.barrier()
+        if rank == 1:
+            time.sleep(2.0)
+        t0 = time.time()
+        J.run(co, 12, 0, use_graph=False)
+        try:
+            co.sync()
+            status = U.UC_OK
+        except U.UCError as e:
+            status = e.status
+        dt = time.time() - t0
+        comm.barrier()
+        J.destroy()
+        co.destroy()
+        comm.destroy()
+        env.finalize()
+        return status, dt
+
+    res = run_ranks(2, body, timeout=60)
+    for status, dt in res:
+        assert status == U.UC_ERR_TIMEOUT and dt < 10.0, res
