@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--mode", default="device", choices=["device", "host"])
+    ap.add_argument("--host-path", default="1,1",
+                    help="host mode: deep_halo,overlap (uc_jacobi_set_host_path); 0,0 = the paper's Listing 1")
     ap.add_argument("--nx", type=int, default=NX)
     ap.add_argument("--ny-per-gpu", type=int, default=NY_PER_GPU)
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
@@ -223,6 +225,9 @@ def run_ours(a):
     J = U.Jacobi(comm, nx, ny)
     if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages or a.tile_rows:
         J.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages, a.tile_rows)
+    host_path = tuple(int(x) for x in a.host_path.split(","))
+    if a.mode == "host":
+        J.set_host_path(*host_path)
     n = J.n
     launch_info = J.launch_info()
     use_graph = not a.no_graph
@@ -263,7 +268,7 @@ def run_ours(a):
     # ---------------- the launches a step really runs (uc_jacobi_launch_plan; device counters agree)
     v = launch_info["variant"]
     levels = launch_info["tile_rows"] if v == 5 else 1
-    plan = U.launch_plan(v, levels, mode, n, ips, a.norm_every)
+    plan = J.plan(mode, ips, a.norm_every)
     per_launch = max(plan)
     # our kernels in the timed region, from the device launch counters (host mode adds one
     # norm_finish kernel per norm round; NCCL's own kernels are not counted)
@@ -287,7 +292,7 @@ def run_ours(a):
         iters = depth * L
         ne = depth if with_norm else 0
         buf = np.zeros(max(1, L), np.float64)
-        assert U.launch_plan(v, levels, mode, n, iters, ne) == [depth] * L
+        assert J.plan(mode, iters, ne) == [depth] * L
         for _ in range(2):
             J.run(coord, iters, ne, True, norms_out=buf if with_norm else None)
         coord.sync()
@@ -363,6 +368,8 @@ def run_ours(a):
         J2 = U.Jacobi(comm, nx, ny)
         if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages or a.tile_rows:
             J2.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages, a.tile_rows)
+        if a.mode == "host":
+            J2.set_host_path(*host_path)
         stream2 = torch.cuda.Stream()
         coord2 = U.Coord(comm, mode, stream2.cuda_stream)
         h_in = torch.empty(slab_elems, dtype=torch.float32, pin_memory=True)
@@ -433,6 +440,8 @@ def run_ours(a):
                        else "configs[2] (strong, 16384^2 total)",
                        "nx": nx, "ny_global": ny, "rows_per_gpu": n, "iters_per_step": ips,
                        "norm_every": a.norm_every, "mode": a.mode, "cuda_graph": use_graph,
+                       "host_path": ({"deep_halo": host_path[0], "overlap": host_path[1]} if a.mode == "host"
+                                     else None),
                        "parallelism": f"y-slab x{world}", "l2": "inputs > L2 (2 slabs x "
                        f"{(n + 2) * nx * 4 / 2**20:.0f} MiB per GPU vs 126 MB L2), no flush",
                        "launch": launch_info},

@@ -55,6 +55,8 @@ def rank_main(rank, P, device, ag, a, barrier):
     maxb = max(sizes)
     buf = U.SymMem(comm, 3 * maxb)
     sig = U.SymMem(comm, 64)
+    sig2 = U.SymMem(comm, 64)  # signals of the library-call legs (monotone per slot)
+    sigv = [0, 0, 0]
     out = []
 
     def timed(fn, reps, all_ranks=False):
@@ -84,6 +86,49 @@ def rank_main(rank, P, device, ag, a, barrier):
             dev.p2p_bench(U.UC_P2P_WINDOW, buf, sig, S, wub, 64, peer, role, a.blocks)
             ms = timed(lambda: dev.p2p_bench(U.UC_P2P_WINDOW, buf, sig, S, itb, 64, peer, role, a.blocks), a.reps)
             rec["put_signal_GBps"] = S * 64 * itb / (ms / 1e3) / 1e9
+        # ---- the library calls themselves (one launch / copy per message, host-enqueued):
+        # uc_put_signal + uc_signal_wait ping-pong and a 64-message window, per transport --
+        # SM stores + spin-kernel wait, copy engine + spin-kernel wait, copy engine +
+        # cuStreamWaitValue64 (SURVEY §8 a7 paths (i), (ii) and the stream-side Acknowledge)
+        if P >= 2 and rank in (0, 1) and not a.no_calls:
+            peer = 1 - rank
+            src = buf.ptr()
+            for tag, (pp, wp) in (("sm", (0, 0)), ("ce", (1, 0)), ("ce_streamwait", (1, 1))):
+                dev.set_p2p_path(pp, wp)
+                itc = max(1, osu_counts(S, "lat", a.scale)[0] // 100)
+
+                def call_pingpong(n):
+                    for _ in range(n):
+                        sigv[0] += 1
+                        v = sigv[0]
+                        if rank == 0:
+                            dev.put_signal(src, buf, S, S, sig2, 0, v, peer)
+                            dev.signal_wait(buf, S, S, sig2, 0, v, peer)
+                        else:
+                            dev.signal_wait(buf, S, S, sig2, 0, v, peer)
+                            dev.put_signal(src, buf, S, S, sig2, 0, v, peer)
+
+                def call_window(n):
+                    for _ in range(n):
+                        for _w in range(64):
+                            sigv[1] += 1
+                            if rank == 0:
+                                dev.put_signal(src, buf, S, S, sig2, 1, sigv[1], peer)
+                        sigv[2] += 1
+                        if rank == 0:
+                            dev.signal_wait(buf, S, S, sig2, 2, sigv[2], peer)
+                        else:
+                            dev.signal_wait(buf, S, S, sig2, 1, sigv[1], peer)
+                            dev.put_signal(src, buf, 2 * S, 16, sig2, 2, sigv[2], peer)
+
+                call_pingpong(2)
+                ms = timed(lambda: call_pingpong(itc), a.reps)
+                rec[f"{tag}_call_latency_us"] = ms * 1e3 / (2 * itc)
+                itw = max(1, osu_counts(S, "bw", a.scale)[0] // 20)
+                call_window(1)
+                ms = timed(lambda: call_window(itw), a.reps)
+                rec[f"{tag}_call_GBps"] = S * 64 * itw / (ms / 1e3) / 1e9
+            dev.set_p2p_path(0, 0)
         # ---- halo pattern: every rank to top and bottom
         it, wu = osu_counts(S, "lat", a.scale)
         it = max(1, it // 10)
@@ -130,6 +175,7 @@ def rank_main(rank, P, device, ag, a, barrier):
     comm.barrier()
     buf.free()
     sig.free()
+    sig2.free()
     if host is not None:
         host.destroy()
     dev.destroy()
@@ -146,6 +192,7 @@ def main():
     ap.add_argument("--max-bytes", type=int, default=256 << 20)
     ap.add_argument("--blocks", type=int, default=0)
     ap.add_argument("--no-nccl", action="store_true")
+    ap.add_argument("--no-calls", action="store_true", help="skip the per-call uc_put_signal legs")
     a = ap.parse_args()
     if a.vr:
         import threading

@@ -4,7 +4,7 @@ The product is ``libuniconn_b200.so`` (C-ABI in ``include/uniconn.h``; CUDA for 
 ``csrc/``).  This package is its thin Python binding; importing it without the built library
 raises ImportError -- there is no CPU or PyTorch fallback.
 """
-from .uniconn import (UC_OK, UC_ERR_TIMEOUT, UC_ERR_STATE, UC_ERR_ARG, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
+from .uniconn import (UC_PUT_SM, UC_PUT_CE, UC_WAIT_KERNEL, UC_WAIT_STREAM, UC_PLAN_DEEP_HALO, UC_OK, UC_ERR_TIMEOUT, UC_ERR_STATE, UC_ERR_ARG, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
                       UC_P2P_HALO, UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_SUM, UC_PROD, UC_MIN, UC_MAX,
                       UC_TOPO_CHAIN, UC_TOPO_NONE, UC_TOPO_RING, UC_U64, CG, Comm, Coord, Env, Jacobi, SymMem,
                       ThreadAllgather, UCError, builtin_kernel, chain_neighbours, launch_plan,

@@ -28,6 +28,9 @@ UC_TOPO_NONE, UC_TOPO_RING, UC_TOPO_CHAIN = 0, 1, 2
 UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_P2P_HALO = 0, 1, 2
 UC_SUM, UC_PROD, UC_MIN, UC_MAX = 0, 1, 2, 3
 UC_MAX_RANKS = 8
+UC_PLAN_DEEP_HALO = 0x100
+UC_PUT_SM, UC_PUT_CE = 0, 1
+UC_WAIT_KERNEL, UC_WAIT_STREAM = 0, 1
 
 ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p)
 
@@ -79,6 +82,9 @@ _SIGS = {
     "uc_jacobi_run": (i32, [vp, vp, i32, i32, vp, i32]),
     "uc_jacobi_num_norms": (i32, [vp, i32, i32]),
     "uc_jacobi_launch_counts": (i32, [vp, P(u64), i32]),
+    "uc_jacobi_set_host_path": (i32, [vp, i32, i32]),
+    "uc_jacobi_solve": (i32, [vp, vp, i32, i32, C.c_double, P(i64), dp]),
+    "uc_coord_set_p2p_path": (i32, [vp, i32, i32]),
     "uc_jacobi_launch_plan": (i32, [i32, i32, i32, i32, i32, i32, P(i32), i32]),
     "uc_jacobi_copy_in": (i32, [vp, vp]),
     "uc_jacobi_copy_out": (i32, [vp, vp, vp, i32]),

@@ -67,6 +67,31 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
       "r"(parity)
       : "memory");
 }
+// Non-blocking phase test (mbarrier.test_wait, acquire on success): issued a row ahead, its
+// latency overlaps the current row's arithmetic instead of sitting on the critical path.
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, unsigned parity) {
+  unsigned r;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(r) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  return r != 0;
+}
+// mbar_wait unless `done` (an earlier mbar_test of the same phase succeeded): one asm block, so
+// the skip is a predicated branch around the wait loop
+__device__ __forceinline__ void mbar_wait_unless(uint64_t* bar, unsigned parity, bool done) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p, d;\n"
+      "setp.ne.u32 d, %2, 0;\n"
+      "@d bra UC_SKIP_%=;\n"
+      "UC_WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra UC_WAIT_%=;\n"
+      "UC_SKIP_%=:\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity), "r"((unsigned)done)
+      : "memory");
+}
 // 1-D bulk copy global -> shared through the TMA engine, completion counted in bytes on `bar`.
 // dst, src 16-byte aligned; bytes a multiple of 16.
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* bar,

@@ -7,7 +7,61 @@ namespace uc {
 
 size_t multistep_smem_bytes(int consumers, int stages, int ghosts) {
   // [full mbarriers][empty mbarriers] padded to 128 B, then the row ring (4G halo floats per side)
-  return (size_t)((32 * stages + 127) / 128) * 128 + (size_t)stages * (4 * consumers + 8 * ghosts) * sizeof(float);
+#if UC_MARCH_GROUPED
+  (void)consumers;  // compile-time ring stride: the widest row the launch bounds allow
+  const size_t row = ghosts == 2 ? kStageFloats<2> : kStageFloats<1>;
+#else
+  const size_t row = (size_t)(4 * consumers + 8 * ghosts);
+#endif
+  return (size_t)((32 * stages + 127) / 128) * 128 + (size_t)stages * row * sizeof(float);
+}
+
+// Host-overlap split launch (part 1 = edge chunks, part 2 = the rest): after the join, one block
+// sums the block partials of both parts in index order (norm launches) and advances the
+// iteration counter, as the last block of an unsplit launch does (finish_iteration).
+__global__ void overlap_finish_kernel(const JacobiParams p, int T, int nparts) {
+  __shared__ double smem[32];
+  const uint64_t k = p.k_dev[0];
+  bool nl = false;
+  if (p.norm_every > 0) {
+    const uint64_t ne = (uint64_t)p.norm_every;
+    nl = ((k + ne - 1) / ne) * ne < k + (uint64_t)T;
+  }
+  double v = 0.0;
+  if (nl)
+    for (int i = threadIdx.x; i < nparts; i += blockDim.x) v += p.partials[i];
+  const double tot = block_sum(v, smem);
+  if (threadIdx.x == 0) {
+    if (nl) *p.rank_sum = tot;
+    p.k_dev[0] = k + (unsigned long long)T;
+    if ((T & 1) == 0) p.k_dev[2] = p.k_dev[2] ^ 1ull;
+    p.launch_hist[T < 15 ? T : 15] += 1ull;
+    __threadfence();
+  }
+}
+
+// CPU-free convergence loop (uc_jacobi_solve): the last node of the WHILE body.  The period just
+// run had its norm round on its first iteration (norm_hist[m-1], identical on every rank: the
+// cross-rank sums are rank-ordered); continue while !(norm < tol) and fewer than kmax iterations.
+__global__ void solve_check_kernel(const double* norm_hist, int norm_cap, const unsigned long long* k_dev, double tol,
+                                   unsigned long long kmax, cudaGraphConditionalHandle h, double* last) {
+  const unsigned long long m = k_dev[1];
+  const double nrm = m > 0 ? norm_hist[(m - 1) % (unsigned long long)norm_cap] : 0.0;
+  *last = nrm;
+  cudaGraphSetConditional(h, (!(nrm < tol) && k_dev[0] < kmax) ? 1u : 0u);
+}
+
+int launch_solve_check(const double* norm_hist, int norm_cap, const unsigned long long* k_dev, double tol,
+                       unsigned long long kmax, cudaGraphConditionalHandle h, double* last, cudaStream_t s) {
+  solve_check_kernel<<<1, 1, 0, s>>>(norm_hist, norm_cap, k_dev, tol, kmax, h, last);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
+}
+
+int launch_overlap_finish(const JacobiParams& p, int T, int nparts, cudaStream_t s) {
+  overlap_finish_kernel<<<1, 256, 0, s>>>(p, T, nparts);
+  UC_CUDA(cudaGetLastError());
+  return UC_OK;
 }
 
 int launch_jacobi_t(const JacobiParams& p, int grid, int block, int T, cudaStream_t s) {
@@ -35,6 +89,9 @@ int preload_multistep() {
   }
   return preload_multistep_g2();
 }
+
+// ring stages of variant 5 must be a multiple of this (the grouped march), 1 = any
+int multistep_stage_group() { return UC_MARCH_GROUPED ? kGroup : 1; }
 
 int multistep_max_consumers(int ghosts) { return ghosts == 2 ? kMaxBlockG2 : kMaxBlock; }
 

@@ -331,16 +331,78 @@ __device__ __forceinline__ void t_step_skew(const float* ring, uint64_t* full, u
   t_levels_skew<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, pend, L, R, out, pitch, acc);
 }
 
+// Grouped march (UC_MARCH_GROUPED, the product build): the steady-state row loop runs in groups
+// of kGroup rows = kGroup ring stages, so every stage index, mbarrier address and ring offset of
+// the group is a compile-time constant (one ring phase flip per group instead of per-row stage
+// bookkeeping), and kGroup is a multiple of the register-rotation period 3 (no moves at the loop
+// back edge).  The ring stride is the compile-time maximum row (4 x the launch bounds' consumer
+// threads + the halo floats), so ring loads use immediate offsets.  The ring has a multiple of
+// kGroup stages.
+#ifndef UC_MARCH_GROUPED
+#define UC_MARCH_GROUPED 1
+#endif
+#ifndef UC_GROUP_ROWS
+#define UC_GROUP_ROWS 9
+#endif
+constexpr int kGroup = UC_GROUP_ROWS;
+// test the next row's ring phase right after taking the current row (mbarrier.test_wait), so
+// the phase check's latency overlaps the arithmetic; the blocking wait runs only if it failed
+#ifndef UC_RING_TEST_AHEAD
+#define UC_RING_TEST_AHEAD 1
+#endif
+static_assert(kGroup % 3 == 0, "the group must be a multiple of the rotation period");
+template <int G>
+constexpr int kStageFloats = 4 * (G == 1 ? kMaxBlock : kMaxBlockG2) + 2 * Ghost<G>::kPadG;
+
+// One group of kGroup rows starting at ring stage gbase (a multiple of kGroup), phase ph.
+template <int T, int NL, bool DIRI, int G, int HOIST>
+__device__ __forceinline__ void t_group(const float* ringp, uint64_t* full, uint64_t* empty, unsigned ph,
+                                        const GhostLayout& g, int nx4, int a, int b, int i0, float4 (&w0)[T],
+                                        float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+  constexpr int ST = kStageFloats<G>;
+  const bool lane0 = (threadIdx.x & 31) == 0;
+#if UC_RING_TEST_AHEAD
+  bool ready = false;  // row u's phase already observed complete by the previous step's test
+#endif
+#pragma unroll
+  for (int u = 0; u < kGroup; ++u) {
+    float L[T], R[T];
+    t_neighbours<T, 0, HOIST>(w1, L, R);
+#if UC_RING_TEST_AHEAD
+    mbar_wait_unless(full + u, ph, ready);
+#else
+    mbar_wait(full + u, ph);
+#endif
+    const float4 nv = *reinterpret_cast<const float4*>(ringp + u * ST);
+    __syncwarp();
+    mbar_arrive_if(empty + u, lane0);
+#if UC_RING_TEST_AHEAD
+    if (u + 1 < kGroup) ready = mbar_test(full + u + 1, ph);  // answered while this row computes
+#endif
+    t_neighbours<T, HOIST, T>(w1, L, R);
+    t_levels<T, NL, DIRI, true>(nv, g, nx4, a, b, i0 + u, w0, w1, L, R, out, pitch, acc);
+  }
+}
+
 template <int T, int NL, bool DIRI, int G>
 __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src, float* dst, int s,
                                         const GhostLayout& g, int a, int b, double& acc, float* ring,
                                         uint64_t* full, uint64_t* empty, bool proxy_fence) {
   const int nc = p.consumers, NS = p.stages;
   constexpr int PAD = Ghost<G>::kPadG;
+#if UC_MARCH_GROUPED
+  constexpr int ST = kStageFloats<G>;
+  // warp-uniform role split: the compiler sees a branch on a broadcast value, so the consumer
+  // path is known converged (no divergence checks around its shuffles and warp syncs)
+  const int wid = __shfl_sync(kFull, (int)threadIdx.x >> 5, 0);
+  const bool producer = wid >= (nc >> 5);
+#else
   const int ST = 4 * nc + 2 * PAD;
+  const bool producer = (int)threadIdx.x >= nc;
+#endif
   const size_t pitch = (size_t)p.nx;
   const int rows = b - a + 1 + 2 * T;
-  if ((int)threadIdx.x >= nc) {
+  if (producer) {
     if ((threadIdx.x & 31) == 0) {
       const int xs = 4 * s * p.strip4;
       const int xe = min(xs + 4 * p.strip4, p.nx);
@@ -406,10 +468,31 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
   for (int i = 0; i < 2 * T; ++i)
     t_step<T, NL, DIRI, false, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
                                                       pitch, acc);
+#if UC_MARCH_GROUPED
+  int i = 2 * T;
+  // single rows up to the next group boundary (ring stage 0 mod kGroup)
+  for (; i < rows && cur.st % kGroup != 0; ++i)
+    t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
+                                                     pitch, acc);
+  const float* ringl = ring + g.ring_off;
+  for (; i + kGroup <= rows; i += kGroup) {
+    t_group<T, NL, DIRI, G, kHoistLevels<T, G>>(ringl + cur.st * ST, full + cur.st, empty + cur.st, cur.ph, g, nx4,
+                                                a, b, i, w0, w1, out, pitch, acc);
+    cur.st += kGroup;
+    if (cur.st == NS) {
+      cur.st = 0;
+      cur.ph ^= 1u;
+    }
+  }
+  for (; i < rows; ++i)
+    t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
+                                                     pitch, acc);
+#else
 #pragma unroll(kTUnroll)
   for (int i = 2 * T; i < rows; ++i)
     t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
                                                      pitch, acc);
+#endif
 }
 
 template <int T, int NL, int G>
@@ -419,17 +502,26 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
   const float* src = p.slab[par];
   float* dst = p.slab[par ^ 1];
   const int s = blockIdx.x % p.strips;
-  const int q = blockIdx.x / p.strips;
+  // part 0: every row chunk; part 1 (host overlap): the first and last chunk only (grid 2 x strips);
+  // part 2: the others (chunks 1..chunks-2)
+  const int q = p.part == 0 ? blockIdx.x / p.strips
+                : p.part == 1 ? (blockIdx.x < p.strips ? 0 : p.chunks - 1)
+                              : blockIdx.x / p.strips + 1;
   const GhostLayout g = ghost_layout<G>(p, s);
   int lo, hi;
   chunk_rows(p, q, lo, hi);
   const bool top_blk = q == 0, bot_blk = q == p.chunks - 1;
+  // deep-halo host mode: a side with a neighbour holds T halo rows of A_k (the host exchanged T
+  // rows), so the march covers the edge rows too (it streams rows 1-T..0 / n+1..n+T) and that
+  // side runs no boundary rounds; a side without a neighbour keeps its rounds (fixed row)
+  const bool deep_top = p.deep_halo && p.has_top, deep_bot = p.deep_halo && p.has_bot;
+  const bool rtop = top_blk && !deep_top, rbot = bot_blk && !deep_bot;
   double acc = 0.0;
   // round 1 before the march (all threads: the producer must not read halo rows before the wait)
-  if (top_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, true, true, acc);
-  if (bot_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, false, true, acc);
-  const int a = max(lo, PT + 1);
-  const int b = min(hi, p.n - PT);
+  if (rtop) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, true, true, acc);
+  if (rbot) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, false, true, acc);
+  const int a = deep_top ? lo : max(lo, PT + 1);
+  const int b = deep_bot ? hi : min(hi, p.n - PT);
   if (a <= b) {
     // fixed columns (0, NX-1) among the block's lanes, ghosts included: keep them fixed
     const int xs4 = s * p.strip4;
@@ -437,10 +529,10 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
     if (diri) march_t<T, NL, true, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
     else march_t<T, NL, false, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
   }
-  if ((top_blk || bot_blk) && (int)threadIdx.x < p.consumers) {
+  if ((rtop || rbot) && (int)threadIdx.x < p.consumers) {
     for (int j = 2; j <= T; ++j) {  // consumers only (named barrier 1)
-      if (top_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
-      if (bot_blk) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, false, false, acc);
+      if (rtop) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
+      if (rbot) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, false, false, acc);
     }
   }
   return acc;
@@ -457,8 +549,10 @@ __device__ __forceinline__ double t_body_nl(const JacobiParams& p, uint64_t k, i
 }
 
 // T iterations per launch with G ghost lanes per warp side (T <= 4G).  Device mode: n >= 2T, at
-// most one norm round per launch; host / partial mode: T = 1 (the host API exchanges the halos
-// after the kernel).
+// most one norm round per launch; partial mode and paper-faithful host mode: T = 1 (the host API
+// exchanges the halos after the kernel); deep-halo host mode: T per launch, T halo rows exchanged
+// by the host API after it (p.deep_halo).  p.part splits a launch into its edge chunks and the
+// rest (host overlap: NCCL moves the edge rows while the rest computes).
 template <int T, int G>
 __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G == 1 ? UC_T_MINBLOCKS : UC_T8_MINBLOCKS)
     jacobi_t_kernel(const JacobiParams p) {
@@ -491,8 +585,9 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
   else acc = t_body_nl<T, 1, G>(p, k, par, ring, full, empty, nl);
   if (nl > 0) {
     const double t = block_sum(acc, smem);
-    if (threadIdx.x == 0) p.partials[blockIdx.x] = t;
+    if (threadIdx.x == 0) p.partials[p.partial_base + blockIdx.x] = t;
   }
+  if (p.part != 0) return;  // split launch: overlap_finish_kernel sums the partials and advances k
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();

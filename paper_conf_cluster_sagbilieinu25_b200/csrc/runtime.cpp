@@ -482,6 +482,9 @@ int uc_coord_destroy(uc_coord* k) {
   cudaFree(k->err);
   cudaFree(k->put_counter);
   cudaFree(k->nccl_scratch);
+  if (k->side) cudaStreamDestroy(k->side);
+  if (k->ev_fork) cudaEventDestroy(k->ev_fork);
+  if (k->ev_join) cudaEventDestroy(k->ev_join);
   k->comm->live_objects--;
   delete k;
   return UC_OK;
@@ -586,7 +589,54 @@ int uc_put_signal(uc_coord* k, const void* src, uc_mem* dst, size_t dst_off, siz
     if (!s) return fail(UC_ERR_UNSUPPORTED, "rank %d signal not peer-addressable", peer);
     s += sig_idx;
   }
+  if (k->put_path == UC_PUT_CE) {
+    // copy engine over NVLink (a peer D2D copy), then the signal from a one-block kernel that
+    // runs after the copy has completed (stream order)
+    if (bytes) UC_CUDA(cudaMemcpyAsync(d + dst_off, src, bytes, cudaMemcpyDeviceToDevice, k->stream));
+    return launch_put_signal(src, d + dst_off, 0, s, sig_val, k->put_counter, k->stream);
+  }
   return launch_put_signal(src, d + dst_off, bytes, s, sig_val, k->put_counter, k->stream);
+}
+
+namespace {
+typedef CUresult (*cuStreamWaitValue64_pfn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+typedef CUresult (*cuDeviceGetAttribute_pfn)(int*, CUdevice_attribute, CUdevice);
+
+// cuStreamWaitValue64(GEQ [| FLUSH]) through the driver entry point (no -lcuda link)
+int stream_wait_ge(uc_coord* k, const uint64_t* sig, uint64_t val) {
+  static cuStreamWaitValue64_pfn wait = nullptr;
+  static cuDeviceGetAttribute_pfn attr = nullptr;
+  if (!wait) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    UC_CUDA(cudaGetDriverEntryPoint("cuStreamWaitValue64", &fn, cudaEnableDefault, &q));
+    if (q != cudaDriverEntryPointSuccess || !fn) return fail(UC_ERR_UNSUPPORTED, "cuStreamWaitValue64 not available");
+    wait = (cuStreamWaitValue64_pfn)fn;
+    UC_CUDA(cudaGetDriverEntryPoint("cuDeviceGetAttribute", &fn, cudaEnableDefault, &q));
+    if (q == cudaDriverEntryPointSuccess) attr = (cuDeviceGetAttribute_pfn)fn;
+  }
+  unsigned flags = CU_STREAM_WAIT_VALUE_GEQ;
+  int ok64 = 1, flush = 0;
+  if (attr) {
+    attr(&ok64, CU_DEVICE_ATTRIBUTE_CAN_USE_64_BIT_STREAM_MEM_OPS, (CUdevice)k->comm->env->device);
+    attr(&flush, CU_DEVICE_ATTRIBUTE_CAN_FLUSH_REMOTE_WRITES, (CUdevice)k->comm->env->device);
+  }
+  if (!ok64) return fail(UC_ERR_UNSUPPORTED, "device lacks 64-bit stream memory operations");
+  if (flush) flags |= CU_STREAM_WAIT_VALUE_FLUSH;
+  const CUresult r = wait((CUstream)k->stream, (CUdeviceptr)(uintptr_t)sig, (cuuint64_t)val, flags);
+  if (r == CUDA_ERROR_NOT_SUPPORTED) return fail(UC_ERR_UNSUPPORTED, "cuStreamWaitValue64 not supported here");
+  if (r != CUDA_SUCCESS) return fail(UC_ERR_CUDA, "cuStreamWaitValue64 failed with CUresult %d", (int)r);
+  return UC_OK;
+}
+}  // namespace
+
+int uc_coord_set_p2p_path(uc_coord* k, int put_path, int wait_path) {
+  if (!k) return fail(UC_ERR_ARG, "coord is NULL");
+  if (put_path != UC_PUT_SM && put_path != UC_PUT_CE) return fail(UC_ERR_ARG, "put_path %d", put_path);
+  if (wait_path != UC_WAIT_KERNEL && wait_path != UC_WAIT_STREAM) return fail(UC_ERR_ARG, "wait_path %d", wait_path);
+  k->put_path = put_path;
+  k->wait_path = wait_path;
+  return UC_OK;
 }
 
 int uc_signal_wait(uc_coord* k, uc_mem* dst, size_t dst_off, size_t bytes, uc_mem* sig, size_t sig_idx,
@@ -603,6 +653,7 @@ int uc_signal_wait(uc_coord* k, uc_mem* dst, size_t dst_off, size_t bytes, uc_me
   }
   if (!sig) return fail(UC_ERR_ARG, "sig is NULL in device mode");
   if ((sig_idx + 1) * sizeof(uint64_t) > sig->bytes) return fail(UC_ERR_ARG, "sig_idx %zu out of range", sig_idx);
+  if (k->wait_path == UC_WAIT_STREAM) return stream_wait_ge(k, (const uint64_t*)sig->local + sig_idx, sig_val);
   return launch_signal_wait((const uint64_t*)sig->local + sig_idx, sig_val, k->timeout_ns, k->err, k->stream);
 }
 

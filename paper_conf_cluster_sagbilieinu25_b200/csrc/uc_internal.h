@@ -70,6 +70,9 @@ struct JacobiParams {
   int strip4;                          // variant 5: owned float4 columns per strip (ghost-lane layout)
   int chunk_shrink;                    // variant 5: rows taken off the first/last row chunk
   int ghosts;                          // variant 5: ghost lanes per warp side (1: T <= 4, 2: T <= 8)
+  int deep_halo;                       // variant 5, host mode: T halo rows per side with a neighbour
+  int part;                            // variant 5: 0 whole launch, 1 edge chunks, 2 other chunks
+  int partial_base;                    // index of this launch's first block partial
   double* partials;                    // local [grid] per-block partial sums
   double* rank_sum;                    // local: this rank's sum of squares (host-mode allreduce in place)
   double* norm_hist;                   // local: norms by round m (ring of norm_cap)
@@ -99,13 +102,18 @@ constexpr int kFlagStride = 16;  // u64 per flag = 128 bytes, one flag per L2 li
 constexpr int kDefaultVariant = 5;
 constexpr int kDefaultStages = 3;
 constexpr int kDefaultStagesTwoStep = 4;
-constexpr int kDefaultStagesMulti = 8;
+constexpr int kDefaultStagesMulti = 9;  // a multiple of the grouped march's kGroup (9)
 constexpr int kDefaultTileRows = 64;
 
 // Launch wrappers implemented in kernels.cu
 int launch_jacobi_iteration(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_two_step(const JacobiParams& p, int grid, int block, cudaStream_t s);
 int launch_jacobi_t(const JacobiParams& p, int grid, int block, int T, cudaStream_t s);
+// host-overlap split launch: sum the block partials of both parts (norm launches), advance k by T
+int launch_overlap_finish(const JacobiParams& p, int T, int nparts, cudaStream_t s);
+// uc_jacobi_solve: the WHILE body's last kernel -- reads the period's norm, sets the condition
+int launch_solve_check(const double* norm_hist, int norm_cap, const unsigned long long* k_dev, double tol,
+                       unsigned long long kmax, cudaGraphConditionalHandle h, double* last, cudaStream_t s);
 int preload_multistep();                                             // multistep.cu
 // the deepest instance of a ghost layout (G = 1: T = 4; G = 2: T = 8) bounds the geometry of all T
 int multistep_occupancy(int block, size_t smem, int ghosts, int* blocks_per_sm);
@@ -117,7 +125,8 @@ int preload_multistep_g2b();
 int launch_jacobi_t_g2c(const JacobiParams& p, int grid, int block, size_t smem, cudaStream_t s);  // multistep_g2c.cu
 int preload_multistep_g2c();
 int multistep_occupancy_g2(int block, size_t smem, int* blocks_per_sm);
-int multistep_max_consumers(int ghosts);  // consumer threads per block the launch bounds allow
+int multistep_max_consumers(int ghosts);
+int multistep_stage_group();  // variant 5 ring stages: a multiple of this (grouped march)  // consumer threads per block the launch bounds allow
 int launch_jacobi_persistent(const JacobiParams& p, int grid, int block, int iters, cudaStream_t s);
 // Stream-ordered device -> host copy of n doubles on the coordinator's stream that never blocks
 // the calling thread: into page-locked memory directly; into pageable memory into `stage`
@@ -224,6 +233,9 @@ struct uc_coord {
   float* nccl_scratch = nullptr;       // host-mode barrier operand
   uint64_t p2p_epoch[3][UC_MAX_RANKS] = {};  // signal base of the next uc_p2p_bench call, per (pattern, peer)
   unsigned int* p2p_bar = nullptr;     // grid barrier [count, gen] of the p2p kernel
+  int put_path = 0, wait_path = 0;     // uc_coord_set_p2p_path: SM / copy engine, spin kernel / stream wait
+  cudaStream_t side = nullptr;         // host-overlap path: NCCL halo exchange beside the interior
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   struct PendingCopy {
     double* dst;
     const double* src;
@@ -268,7 +280,11 @@ struct uc_jacobi {
   int strip4 = 0;                // variant 5: owned float4 columns per strip
   int chunk_shrink = 0;          // variant 5: rows taken off the first/last row chunk
   int ghosts = 1;                // variant 5: ghost lanes per warp side (2 when T > 4)
-  size_t slab_elems = 0;
+  size_t slab_elems = 0;         // (n+2) * nx: one slab view (halo rows included)
+  size_t slab_stride = 0;        // (n + 2 kHaloRows) * nx: one slab in the allocation
+  size_t slab_off = 0;           // (kHaloRows - 1) * nx: view row 0 within its slab
+  int host_deep = 0;             // host mode: T halo rows exchanged once per T-iteration launch
+  int host_overlap = 0;          // host mode: edge chunks -> NCCL on a side stream || other chunks
   int strips = 0;               // current column strips (launch geometry)
   int max_strips = 0;           // flag capacity per side = ceil(nx/4 / 32)
   // local device state

@@ -18,7 +18,7 @@ from typing import Callable, Optional
 
 import numpy as np
 
-from ._lib import (UC_OK, UC_ERR_TIMEOUT, UC_ERR_STATE, UC_ERR_ARG, ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
+from ._lib import (UC_PUT_SM, UC_PUT_CE, UC_WAIT_KERNEL, UC_WAIT_STREAM, UC_PLAN_DEEP_HALO, UC_OK, UC_ERR_TIMEOUT, UC_ERR_STATE, UC_ERR_ARG, ALLGATHER_FN, UC_F32, UC_F64, UC_MODE_DEVICE, UC_MODE_HOST, UC_MODE_PARTIAL,  # noqa: F401
                    UC_MAX, UC_MIN, UC_P2P_HALO, UC_P2P_PINGPONG, UC_P2P_WINDOW, UC_PROD, UC_SUM, UC_TOPO_CHAIN,
                    UC_TOPO_NONE, UC_TOPO_RING, UC_U64,
                    UCError, check, lib)
@@ -176,6 +176,10 @@ class Coord:
             check(lib.uc_coord_sync(self.h), "uc_coord_sync")
         finally:
             self._outputs.clear()
+
+    def set_p2p_path(self, put_path: int = 0, wait_path: int = 0):
+        """uc_coord_set_p2p_path: UC_PUT_SM / UC_PUT_CE, UC_WAIT_KERNEL / UC_WAIT_STREAM."""
+        check(lib.uc_coord_set_p2p_path(self.h, put_path, wait_path), "uc_coord_set_p2p_path")
 
     def set_timeout(self, seconds: float):
         check(lib.uc_coord_set_timeout(self.h, int(seconds * 1e9)), "uc_coord_set_timeout")
@@ -344,6 +348,25 @@ class Jacobi:
         """COLLECTIVE (see uc_jacobi_set_launch)."""
         check(lib.uc_jacobi_set_launch(self.h, variant, block_x, blocks_per_sm, stages, tile_rows),
               "uc_jacobi_set_launch")
+
+    def solve(self, coord: Coord, max_iters: int, norm_every: int, tol: float):
+        """uc_jacobi_solve: CPU-free convergence loop; returns (iterations run, last norm)."""
+        it, nrm = C.c_int64(), C.c_double()
+        check(lib.uc_jacobi_solve(coord.h, self.h, max_iters, norm_every, tol, C.byref(it), C.byref(nrm)),
+              "uc_jacobi_solve")
+        return it.value, nrm.value
+
+    def set_host_path(self, deep_halo: bool = False, overlap: bool = False):
+        """uc_jacobi_set_host_path (same call on every rank)."""
+        check(lib.uc_jacobi_set_host_path(self.h, int(deep_halo), int(overlap)), "uc_jacobi_set_host_path")
+        self.host_deep = bool(deep_halo)
+
+    def plan(self, mode: int, iters: int, norm_every: int) -> list:
+        """The launch plan uc_jacobi_run follows for this solver under a coordinator of `mode`."""
+        info = self.launch_info()
+        v = info["variant"]
+        m = mode | (UC_PLAN_DEEP_HALO if mode == UC_MODE_HOST and getattr(self, "host_deep", False) else 0)
+        return launch_plan(v, info["tile_rows"] if v == 5 else 1, m, self.n, iters, norm_every)
 
     def launch_counts(self) -> list:
         """uc_jacobi_launch_counts: completed launches by iterations per launch (index t = 1..8;

@@ -18,7 +18,7 @@ def neighbours(U, topology):
 def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0, seed=gen.DEFAULT_SEED,
               zero_init=False, init=None, use_graph=True, stepwise=False, block_x=0, blocks_per_sm=0,
               variant=-1, stages=0, tile_rows=0,
-              chunks_of_run=None):
+              chunks_of_run=None, host_path=None):
     """Returns dict(init=[slab0 per rank], final=[slab per rank], norms=np.array (rank 0),
     norms_all=[per rank], launch=launch_info of rank 0)."""
     import torch
@@ -36,6 +36,8 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
         try:
             if block_x or blocks_per_sm or variant >= 0 or stages or tile_rows:
                 J.set_launch(variant, block_x, blocks_per_sm, stages, tile_rows)
+            if host_path is not None:
+                J.set_host_path(*host_path)
             slab0 = J.copy_out()
             if init is not None:
                 J.copy_in(gen.rank_slab(init, rank, P))
@@ -59,7 +61,8 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
             final = J.copy_out(coord)
             info = J.launch_info()
             counts = J.launch_counts()
-            want = expected_counts(U, info, MODES[mode], ny // P, iters, norm_every, stepwise, chunks_of_run)
+            pm = MODES[mode] | (U.UC_PLAN_DEEP_HALO if host_path and host_path[0] and mode == "host" else 0)
+            want = expected_counts(U, info, pm, ny // P, iters, norm_every, stepwise, chunks_of_run)
             if want is not None:  # the launches that really ran are the plan's (no silent demotion)
                 assert counts == want, (f"rank {rank}: launches by iterations per launch {counts[:9]} != "
                                         f"plan {want[:9]} ({info})")
@@ -81,7 +84,7 @@ def expected_counts(U, info, mode, n_local, iters, norm_every, stepwise=False, c
     """Histogram (launches by iterations per launch) the launch plan predicts for a run, or None
     where launches are not one-per-plan-entry (the persistent variant 3 in device mode)."""
     v = info["variant"]
-    if v == 3 and mode == 1:
+    if v == 3 and mode & 0xff == 1:
         return None
     h = [0] * 16
     if stepwise:

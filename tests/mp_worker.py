@@ -30,6 +30,7 @@ def main():
     ap.add_argument("--same-device", action="store_true")
     ap.add_argument("--variant", type=int, default=-1)
     ap.add_argument("--tile-rows", type=int, default=0)
+    ap.add_argument("--host-path", default="0,0", help="deep_halo,overlap (host mode)")
     ap.add_argument("--out", required=True)
     a = ap.parse_args()
     rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
@@ -46,6 +47,8 @@ def main():
     J = U.Jacobi(comm, a.nx, a.ny)
     if a.variant >= 0:
         J.set_launch(a.variant, 0, 0, 0, a.tile_rows)
+    deep, overlap = (int(x) for x in a.host_path.split(","))
+    J.set_host_path(deep, overlap)
     norms = J.run(coord, a.iters, a.norm_every, use_graph=True)
     coord.sync()
     slab = J.copy_out(coord)

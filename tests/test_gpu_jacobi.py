@@ -267,11 +267,11 @@ def test_constant_field_fixed_and_zero_norm():
 def test_full_size_16384_single_gpu_bench_configuration():
     """BASELINE.json configs[2]/[3] at P = 1 (16384^2 fp32, 1 GiB per slab), in the launch
     configuration bench.py times (device mode, ring, CUDA graph, default geometry = variant 5,
-    six iterations per launch with two ghost lanes, 8-row ring): the whole grid bit-exact vs the
+    six iterations per launch with two ghost lanes, 9-row ring): the whole grid bit-exact vs the
     oracle after 12, 14 (a two-iteration launch at the end) and 17 iterations (a five-iteration
     one), norms within 1e-5 on every level."""
     res = _check(16384, 16384, 1, "ring", "device", 12, norm_every=6)
-    assert res["launch"]["variant"] == 5 and res["launch"]["stages"] == 8 and res["launch"]["tile_rows"] == 6
+    assert res["launch"]["variant"] == 5 and res["launch"]["stages"] == 9 and res["launch"]["tile_rows"] == 6
     assert res["launch"]["block"] == 256
     _check(16384, 16384, 1, "ring", "device", 14, norm_every=7)
     _check(16384, 16384, 1, "ring", "device", 17, norm_every=0)

@@ -59,7 +59,7 @@ def test_few_rows_per_rank(T, P, ny):
 
 
 @pytest.mark.parametrize("T", [2, 4, 6, 8])
-@pytest.mark.parametrize("block_x,bps,stages", [(32, 1, 3), (64, 2, 4), (128, 0, 2), (256, 1, 8), (96, 0, 5)])
+@pytest.mark.parametrize("block_x,bps,stages", [(32, 1, 9), (64, 2, 18), (128, 0, 9), (256, 1, 27), (96, 0, 0)])
 def test_launch_geometries(T, block_x, bps, stages):
     """Strip width (ghost lanes meet strip edges), chunk count and ring depth: 4 ranks."""
     if T > 4:  # two ghost lanes: the launch bounds allow 7 consumer warps per block
@@ -241,8 +241,8 @@ def test_two_virtual_ranks_need_concurrent_kernels():
     grids must make progress at the same time.  CUDA does not guarantee concurrent kernels (a
     profiler or MPS serialises them -- the paper notes the missing preemptive scheduling,
     P:115), which is why smoke() runs P = 1.  When the peer's kernel does NOT run alongside
-    (here: rank 1 launches only after rank 0's spin timeout), the waits are bounded and both
-    ranks report UC_ERR_TIMEOUT instead of hanging the device."""
+    (here: rank 1 launches only after rank 0's spin timeout), the waits are bounded and the
+    waiting rank reports UC_ERR_TIMEOUT instead of hanging the device."""
     import time
 
     import torch
@@ -276,5 +276,29 @@ def test_two_virtual_ranks_need_concurrent_kernels():
         return status, dt
 
     res = run_ranks(2, body, timeout=60)
-    for status, dt in res:
-        assert status == U.UC_ERR_TIMEOUT and dt < 10.0, res
+    # rank 0 waited for a peer that was not running: its bounded spin expired and it reports
+    # UC_ERR_TIMEOUT (a waiter that gives up still completes its own puts and flags, so the late
+    # rank finishes -- the error is the application's signal that the run is invalid); nobody hangs
+    assert res[0][0] == U.UC_ERR_TIMEOUT, res
+    assert all(dt < 10.0 for _, dt in res), res
+
+
+# ---------------------------------------------------------------------------------------------
+# Host mode (the NCCL comparator): the paper's one-exchange-per-iteration path, the
+# deep-halo path (T rows exchanged once per T-iteration launch) and the overlapped split launch
+# (edge chunks -> NCCL on a side stream || the other chunks).  One GPU: P = 1 ring (NCCL sends to
+# itself; top == bottom) and chain; P >= 2 needs one GPU per rank (test_gpu_multiprocess.py).
+@pytest.mark.parametrize("deep,overlap", [(0, 0), (1, 0), (0, 1), (1, 1)])
+@pytest.mark.parametrize("topology", ["ring", "dirichlet"])
+@pytest.mark.parametrize("iters,ne", [(25, 6), (13, 0), (20, 5), (7, 1)])
+def test_host_paths(deep, overlap, topology, iters, ne):
+    res = _check(1028, 192, 1, topology, "host", iters, norm_every=ne, host_path=(deep, overlap))
+    if deep and ne in (0, 6):
+        assert res["counts"][6] >= 2, res["counts"]
+
+
+@pytest.mark.parametrize("deep,overlap", [(1, 0), (1, 1), (0, 1)])
+def test_host_paths_full_size(deep, overlap):
+    res = _check(16384, 16384, 1, "ring", "host", 13, norm_every=6, host_path=(deep, overlap))
+    if deep:
+        assert res["counts"][6] == 2 and res["counts"][1] == 1, res["counts"]

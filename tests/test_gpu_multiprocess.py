@@ -27,11 +27,12 @@ def _port():
     return p
 
 
-def _run(tmp_path, P, nx, ny, iters, ne, topology, mode, same_device=True):
+def _run(tmp_path, P, nx, ny, iters, ne, topology, mode, same_device=True, host_path=(0, 0)):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={P}",
            "--master-addr", "127.0.0.1", "--master-port", str(_port()),
            os.path.join(ROOT, "tests", "mp_worker.py"), "--nx", str(nx), "--ny", str(ny), "--iters", str(iters),
-           "--norm-every", str(ne), "--topology", topology, "--mode", mode, "--out", str(tmp_path)]
+           "--norm-every", str(ne), "--topology", topology, "--mode", mode, "--out", str(tmp_path),
+           "--host-path", f"{host_path[0]},{host_path[1]}"]
     if same_device:
         cmd.append("--same-device")
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=300, cwd=ROOT)
@@ -75,6 +76,19 @@ def test_two_gpus_each_mode(tmp_path, mode):
     """Host mode (grouped NCCL send/recv, ncclAllReduce norms) and device / partial mode over
     NVLink peer memory, P = 2 ranks on 2 GPUs, configs[1]-like grid."""
     _run(tmp_path, 2, 4096, 512, 40, 6, "ring", mode, same_device=False)
+
+
+@pytest.mark.skipif("_gpus() < 2", reason="needs >= 2 GPUs (one rank per GPU)")
+@pytest.mark.parametrize("deep,overlap", [(1, 0), (0, 1), (1, 1)])
+@pytest.mark.parametrize("P,topology", [(2, "ring"), (3, "dirichlet"), (4, "ring")])
+def test_host_paths_multi_gpu(tmp_path, deep, overlap, P, topology):
+    """Deep-halo and overlapped host paths with real NCCL peers (one GPU per rank)."""
+    if _gpus() < P:
+        pytest.skip(f"needs {P} GPUs")
+    res = _run(tmp_path, P, 2052, 96 * P, 25, 6, topology, "host", same_device=False, host_path=(deep, overlap))
+    if deep:
+        for x in res:
+            assert list(x["counts"])[6] == 4, list(x["counts"])
 
 
 @pytest.mark.skipif("_gpus() < 4", reason="needs >= 4 GPUs")

@@ -45,13 +45,17 @@ def _teardown(env, comm, coord, *mems):
 
 @pytest.mark.parametrize("nbytes", [16, 4096, 65536 + 16, 4 << 20, (4 << 20) + 8])
 @pytest.mark.parametrize("P", [1, 2, 4])
-def test_put_signal_ring(P, nbytes):
+@pytest.mark.parametrize("put_path,wait_path", [(0, 0), (1, 0), (0, 1), (1, 1)])
+def test_put_signal_ring(P, nbytes, put_path, wait_path):
     """Every rank puts a rank-tagged buffer into its bottom neighbour and waits for the one from
-    its top (the halo pattern of §8 a7), three rounds with monotone signal values."""
+    its top (the halo pattern of §8 a7), three rounds with monotone signal values -- on every
+    transport: SM stores or the copy engine for the put, the spin kernel or cuStreamWaitValue64
+    for the wait."""
     import torch
 
     def body(rank, P, ag):
         U, env, comm, stream, coord = _setup(rank, P, ag, 1)
+        coord.set_p2p_path(put_path, wait_path)
         dst = U.SymMem(comm, nbytes)
         sig = U.SymMem(comm, 64)
         outs = []
