@@ -132,18 +132,21 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
   const bool dev = p.device_mode == 1;
   const size_t pitch = (size_t)p.nx;
   const int side = top ? 0 : 1;          // our h rows: 0 = from top, 1 = from bottom
-  if (threadIdx.x == 0 && has && dev) {
-    if (j == 1) wait_strip_flags(p, top ? 0 : p.flag_half, s, k);  // A_k halo rows
+  // warp 0 waits (all its lanes, warp-uniform loops: keeps the march after round 1 provably
+  // converged), the block follows at the barrier
+  const int wid = warp_id_uniform();
+  if (wid == 0 && has && dev) {
+    if (j == 1) wait_strip_flags_warp(p, top ? 0 : p.flag_half, s, k);  // A_k halo rows
     else {  // the neighbour's level j-1 edge row (its round j-1)
       const uint64_t* f = p.h1_flags + (size_t)(j - 2) * 2 * p.flag_half * kFlagStride;
       const int base = top ? 0 : p.flag_half;
       const int s0 = s > 0 ? s - 1 : 0, s1 = s + 1 < p.strips ? s + 1 : s;
-      for (int q = s0; q <= s1; ++q) wait_ge(f + (size_t)(base + q) * kFlagStride, k + j - 1, p.timeout_ns, p.err);
+      for (int q = s0; q <= s1; ++q) wait_ge_warp(f + (size_t)(base + q) * kFlagStride, k + j - 1, p.timeout_ns, p.err);
     }
   }
   if (cta_sync) __syncthreads();
   else named_barrier_sync(1, p.consumers);
-  if ((int)threadIdx.x >= p.consumers) return;  // the producer warp (cta_sync rounds only)
+  if (wid >= (p.consumers >> 5)) return;  // the producer warp (cta_sync rounds only)
   float4 a[NR];
 #pragma unroll
   for (int i = 0; i < NR; ++i) {
@@ -187,16 +190,17 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
   }
   if (has && dev) {
     named_barrier_sync(1, p.consumers);
-    if (threadIdx.x == 0) {
+    if (wid == 0) {
       __threadfence_system();
-      if (j < T) {
-        uint64_t* f = (top ? p.top_h1_flags : p.bot_h1_flags) + (size_t)(j - 1) * 2 * p.flag_half * kFlagStride;
-        st_release_sys(f + (size_t)((top ? p.flag_half : 0) + s) * kFlagStride, k + j);
-      } else if (top) {
-        st_release_sys(p.top_flags + (size_t)(p.flag_half + s) * kFlagStride, k + T);  // top's from_bottom[s]
-      } else {
-        st_release_sys(p.bot_flags + (size_t)s * kFlagStride, k + T);                  // bottom's from_top[s]
-      }
+      uint64_t* f;
+      if (j < T)
+        f = (top ? p.top_h1_flags : p.bot_h1_flags) + (size_t)(j - 1) * 2 * p.flag_half * kFlagStride +
+            (size_t)((top ? p.flag_half : 0) + s) * kFlagStride;
+      else if (top)
+        f = p.top_flags + (size_t)(p.flag_half + s) * kFlagStride;  // top's from_bottom[s]
+      else
+        f = p.bot_flags + (size_t)s * kFlagStride;                  // bottom's from_top[s]
+      if ((threadIdx.x & 31) == 0) st_release_sys(f, j < T ? k + j : k + T);
     }
   }
 }
@@ -421,7 +425,12 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
       for (int i = 0; i < rows; ++i) {
         if (i >= NS) mbar_wait(empty + st, ph ^ 1u);
         mbar_arrive_expect_tx(full + st, bytes);
+#ifdef UC_PROTO_L2_ROWS  // A/B measurement only (scripts/proto): cycle over a few L2-resident rows
+        bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(a - T + i % UC_PROTO_L2_ROWS) * pitch + left, bytes,
+                 full + st, pol);
+#else
         bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(a - T + i) * pitch + left, bytes, full + st, pol);
+#endif
         if (++st == NS) {
           st = 0;
           ph ^= 1u;
@@ -495,6 +504,23 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
 #endif
 }
 
+// Boundary rounds 2..T after the march, out of line: the march's register allocation then does not
+// carry the rounds' state (their row window, the block's geometry) across its loop.
+#ifndef UC_ROUNDS_NOINLINE
+#define UC_ROUNDS_NOINLINE 0  // A/B: out of line spills more (0.4131 vs 0.4086 ms, scripts/proto)
+#endif
+template <int T, int NL, int G>
+__device__ __noinline__ double t_rounds_after(const JacobiParams& p, const float* src, float* dst, int par, int s,
+                                              uint64_t k, bool rtop, bool rbot) {
+  const GhostLayout g = ghost_layout<G>(p, s);
+  double acc = 0.0;
+  for (int j = 2; j <= T; ++j) {  // consumers only (named barrier 1)
+    if (rtop) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
+    if (rbot) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, false, false, acc);
+  }
+  return acc;
+}
+
 template <int T, int NL, int G>
 __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int par, float* ring, uint64_t* full,
                                          uint64_t* empty) {
@@ -530,10 +556,14 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
     else march_t<T, NL, false, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
   }
   if ((rtop || rbot) && (int)threadIdx.x < p.consumers) {
+#if UC_ROUNDS_NOINLINE
+    acc += t_rounds_after<T, NL, G>(p, src, dst, par, s, k, rtop, rbot);
+#else
     for (int j = 2; j <= T; ++j) {  // consumers only (named barrier 1)
       if (rtop) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
       if (rbot) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, false, false, acc);
     }
+#endif
   }
   return acc;
 }
@@ -555,7 +585,7 @@ __device__ __forceinline__ double t_body_nl(const JacobiParams& p, uint64_t k, i
 // rest (host overlap: NCCL moves the edge rows while the rest computes).
 template <int T, int G>
 __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G == 1 ? UC_T_MINBLOCKS : UC_T8_MINBLOCKS)
-    jacobi_t_kernel(const JacobiParams p) {
+    jacobi_t_kernel(const __grid_constant__ JacobiParams p) {
   static_assert(T >= 1 && T <= 4 * G, "a ghost lane covers 4 levels");
   __shared__ double smem[32];
   __shared__ int s_last;
@@ -580,6 +610,10 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
     const uint64_t first = ((k + ne - 1) / ne) * ne;
     if (first < k + T) nl = (int)(first - k) + 1;
   }
+  // the same in every thread, but loaded from memory: broadcast it so the compiler knows the
+  // NL dispatch below is warp-uniform (otherwise every shuffle of the march gets a divergence
+  // check and every ring wait a reconvergence region)
+  nl = __shfl_sync(kFull, nl, 0);
   double acc = 0.0;
   if (nl == 0) t_body<T, 0, G>(p, k, par, ring, full, empty);
   else acc = t_body_nl<T, 1, G>(p, k, par, ring, full, empty, nl);

@@ -142,6 +142,35 @@ __device__ __forceinline__ void wait_strip_flags(const JacobiParams& p, int base
   for (int j = s0; j <= s1; ++j) wait_ge(p.my_flags + (size_t)(base + j) * kFlagStride, v, p.timeout_ns, p.err);
 }
 
+// The same waits executed by ALL 32 lanes of one warp, with warp-vote loop conditions: the loop is
+// provably warp-uniform, so the code after it stays provably converged (a single-thread spin
+// loop makes the compiler guard every later shuffle with a divergence check and every later
+// mbarrier wait with a reconvergence region -- ~10 % more instructions in the march).
+__device__ __forceinline__ bool wait_ge_warp(const uint64_t* sig, uint64_t v, unsigned long long timeout_ns,
+                                             unsigned int* err) {
+  if (__all_sync(kFull, uc_dev_ld_acquire(sig) >= v)) return true;
+  const unsigned long long t0 = uc_dev_globaltimer();
+  unsigned ns = 32;
+  while (!__all_sync(kFull, uc_dev_ld_relaxed(sig) >= v)) {
+    const bool give_up = uc_dev_globaltimer() - t0 > timeout_ns || *(volatile unsigned int*)err;
+    if (__any_sync(kFull, give_up)) {
+      if ((threadIdx.x & 31) == 0) atomicOr(err, 1u);
+      return false;
+    }
+    __nanosleep(ns);
+    if (ns < 256) ns <<= 1;
+  }
+  asm volatile("fence.acq_rel.sys;" ::: "memory");  // the observing load + fence = acquire
+  return true;
+}
+__device__ __forceinline__ void wait_strip_flags_warp(const JacobiParams& p, int base, int s, uint64_t v) {
+  const int s0 = s > 0 ? s - 1 : 0;
+  const int s1 = s + 1 < p.strips ? s + 1 : s;
+  for (int j = s0; j <= s1; ++j) wait_ge_warp(p.my_flags + (size_t)(base + j) * kFlagStride, v, p.timeout_ns, p.err);
+}
+// warp index, broadcast from lane 0: branches on it are known warp-uniform
+__device__ __forceinline__ int warp_id_uniform() { return __shfl_sync(kFull, (int)threadIdx.x >> 5, 0); }
+
 // ------------------------------------------------------------------------------ reductions
 __device__ __forceinline__ double block_sum(double v, double* smem) {
 #pragma unroll

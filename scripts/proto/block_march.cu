@@ -47,6 +47,11 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
   chunk_rows(p, q, lo, hi);
   const int a = max(lo, T + 1), b = min(hi, p.n - T);
   double acc = 0.0;
+#ifdef PROTO_R1
+  const uint64_t k = p.k_dev[0];
+  const int par = (int)((k + p.k_dev[2]) & 1);
+  if (q == 0) t_round<T, 0>(p, p.slab[par], p.slab[par ^ 1], par ^ 1, s, g, k, 1, true, true, acc);
+#endif
   if (a <= b) {
     const int xs4 = s * p.strip4;
     const bool diri = xs4 <= 1 || xs4 + p.strip4 >= p.nx4 - 1;
@@ -121,7 +126,44 @@ int main(int argc, char** argv) {
     s = d;
     d = x;
   }
-  kern<<<grid, nc + 32, smem>>>(p);
+#ifdef PROTO_FULL
+  // the product kernel itself, P = 1 dirichlet chain (boundary rounds with fixed halo rows, no
+  // waits, no puts), the product's chunk shrink
+  unsigned long long *k_dev, *hist;
+  unsigned int* done;
+  double *parts, *rsum, *nh;
+  CK(cudaMalloc(&k_dev, 64));
+  CK(cudaMemset(k_dev, 0, 64));
+  CK(cudaMalloc(&hist, 128));
+  CK(cudaMemset(hist, 0, 128));
+  CK(cudaMalloc(&done, 64));
+  CK(cudaMemset(done, 0, 64));
+  CK(cudaMalloc(&parts, 8 * 4096));
+  CK(cudaMalloc(&rsum, 64));
+  CK(cudaMalloc(&nh, 8 * 4096));
+  p.k_dev = k_dev;
+  p.launch_hist = hist;
+  p.done = done;
+  p.work = done + 1;
+  p.nbar = done + 2;
+  p.partials = parts;
+  p.rank_sum = rsum;
+  p.norm_hist = nh;
+  p.norm_cap = 4096;
+  p.device_mode = 1;
+  p.size = 1;
+  p.flag_half = strips;
+  int shrink = getenv("PROTO_SHRINK") ? atoi(getenv("PROTO_SHRINK")) : (T > 4 ? 80 * (T - 2) : 40 * T);
+  while (shrink > 0 && (n + 2 * shrink) / chunks - shrink < T + 1) --shrink;
+  p.chunk_shrink = shrink;
+  auto fk = jacobi_t_kernel<PROTO_T, PROTO_G>;
+  CK(cudaFuncSetAttribute(fk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  CK(cudaFuncGetAttributes(&fa, fk));
+#define KLAUNCH fk<<<grid, nc + 32, smem>>>(p)
+#else
+#define KLAUNCH kern<<<grid, nc + 32, smem>>>(p)
+#endif
+  KLAUNCH;
   CK(cudaGetLastError());
   CK(cudaDeviceSynchronize());
   std::vector<unsigned> hb(cnt), hr(cnt);
@@ -136,10 +178,10 @@ int main(int argc, char** argv) {
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);
-  for (int w = 0; w < 3; ++w) kern<<<grid, nc + 32, smem>>>(p);
+  for (int w = 0; w < 3; ++w) KLAUNCH;
   const int reps = 20;
   cudaEventRecord(e0);
-  for (int r = 0; r < reps; ++r) kern<<<grid, nc + 32, smem>>>(p);
+  for (int r = 0; r < reps; ++r) KLAUNCH;
   cudaEventRecord(e1);
   CK(cudaEventSynchronize(e1));
   float ms = 0;
@@ -147,8 +189,8 @@ int main(int argc, char** argv) {
   ms /= reps;
   const double pts = (double)n * (nx - 2);
   printf("{\"tag\": \"%s\", \"T\": %d, \"G\": %d, \"warps\": %d, \"NS\": %d, \"regs\": %d, \"spill\": %d, \"bps\": %d, "
-         "\"grid\": %d, \"strips\": %d, \"chunks\": %d, \"ms\": %.5f, \"GBs\": %.1f, \"glups\": %.1f, \"bad\": %zu}\n",
-         argc > 6 ? argv[6] : "", T, G, warps, NS, fa.numRegs, (int)fa.localSizeBytes, bps, grid, strips, chunks, ms,
+         "\"grid\": %d, \"strips\": %d, \"chunks\": %d, \"shrink\": \"%s\", \"ms\": %.5f, \"GBs\": %.1f, \"glups\": %.1f, \"bad\": %zu}\n",
+         argc > 6 ? argv[6] : "", T, G, warps, NS, fa.numRegs, (int)fa.localSizeBytes, bps, grid, strips, chunks, getenv("PROTO_SHRINK") ? getenv("PROTO_SHRINK") : "-", ms,
          8.0 * pts / (ms * 1e-3) / 1e9, pts * T / (ms * 1e-3) / 1e9, bad);
   return bad ? 2 : 0;
 }
