@@ -56,7 +56,24 @@ __device__ __forceinline__ void mbar_arrive_if(uint64_t* bar, bool pred) {
       "r"((unsigned)pred)
       : "memory");
 }
+// UC_WAIT_HINT_NS > 0: try_wait's suspend-time hint -- the waiting warp sleeps up to that long in
+// ONE try_wait (woken when the phase completes) instead of re-issuing try_wait + branch in a
+// loop, which takes issue slots from the warps that have work
+#ifndef UC_WAIT_HINT_NS
+#define UC_WAIT_HINT_NS 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
+#if UC_WAIT_HINT_NS > 0
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "UC_WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
+      "@!p bra UC_WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity), "n"(UC_WAIT_HINT_NS)
+      : "memory");
+#else
   asm volatile(
       "{\n"
       ".reg .pred p;\n"
@@ -66,6 +83,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
       "}\n" ::"r"(smem_u32(bar)),
       "r"(parity)
       : "memory");
+#endif
 }
 // Non-blocking phase test (mbarrier.test_wait, acquire on success): issued a row ahead, its
 // latency overlaps the current row's arithmetic instead of sitting on the critical path.
@@ -85,11 +103,15 @@ __device__ __forceinline__ void mbar_wait_unless(uint64_t* bar, unsigned parity,
       "setp.ne.u32 d, %2, 0;\n"
       "@d bra UC_SKIP_%=;\n"
       "UC_WAIT_%=:\n"
+#if UC_WAIT_HINT_NS > 0
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %3;\n"
+#else
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+#endif
       "@!p bra UC_WAIT_%=;\n"
       "UC_SKIP_%=:\n"
       "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity), "r"((unsigned)done)
+      "r"(parity), "r"((unsigned)done), "n"(UC_WAIT_HINT_NS > 0 ? UC_WAIT_HINT_NS : 1)
       : "memory");
 }
 // 1-D bulk copy global -> shared through the TMA engine, completion counted in bytes on `bar`.

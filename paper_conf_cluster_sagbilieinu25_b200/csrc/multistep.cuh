@@ -6,6 +6,30 @@
 
 namespace uc {
 
+// A/B instrumentation only (build.py --define UC_TRACE=1 --out ...): %globaltimer stamps per block
+// of the deep-T launches (kernel start, after round 1, after the march, after each later round,
+// end) into a managed buffer the host reads with uc_debug_trace_buffer().  Off in the product.
+#ifndef UC_TRACE
+#define UC_TRACE 0
+#endif
+#if UC_TRACE
+static __device__ unsigned long long* uc_trace_ptr;
+#define UC_TRACE_AT(slot)                                                                       \
+  do {                                                                                         \
+    if (threadIdx.x == 0 && uc_trace_ptr) uc_trace_ptr[blockIdx.x * 16 + (slot)] = globaltimer(); \
+  } while (0)
+#else
+#define UC_TRACE_AT(slot) \
+  do {                    \
+  } while (0)
+#endif
+
+// System-scope fence before the release-store of a round's flag to a neighbour on another GPU
+// (A/B: 0 relies on st.release.sys cumulativity after the block barrier alone)
+#ifndef UC_ROUND_SYS_FENCE
+#define UC_ROUND_SYS_FENCE 1
+#endif
+
 // ------------------------------------------------------------------------------ T iterations per launch
 // Variant 5: one launch advances A_k -> A_{k+T}, T = 1..8 (temporal blocking of depth T).  The
 // staged march keeps T register levels: from the A_k row r streamed through the TMA ring it
@@ -141,7 +165,8 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
       const uint64_t* f = p.h1_flags + (size_t)(j - 2) * 2 * p.flag_half * kFlagStride;
       const int base = top ? 0 : p.flag_half;
       const int s0 = s > 0 ? s - 1 : 0, s1 = s + 1 < p.strips ? s + 1 : s;
-      for (int q = s0; q <= s1; ++q) wait_ge_warp(f + (size_t)(base + q) * kFlagStride, k + j - 1, p.timeout_ns, p.err);
+      for (int q = s0; q <= s1; ++q)
+        wait_ge_warp(f + (size_t)(base + q) * kFlagStride, k + j - 1, p.timeout_ns, p.err, p.gpu_scope != 0);
     }
   }
   if (cta_sync) __syncthreads();
@@ -191,7 +216,12 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
   if (has && dev) {
     named_barrier_sync(1, p.consumers);
     if (wid == 0) {
-      __threadfence_system();
+      // the block's row stores (ordered before this warp by the barrier) become visible before
+      // the flag: a fence at the protocol's scope, then the release store
+      if (p.gpu_scope) __threadfence();
+#if UC_ROUND_SYS_FENCE
+      else __threadfence_system();
+#endif
       uint64_t* f;
       if (j < T)
         f = (top ? p.top_h1_flags : p.bot_h1_flags) + (size_t)(j - 1) * 2 * p.flag_half * kFlagStride +
@@ -200,7 +230,10 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
         f = p.top_flags + (size_t)(p.flag_half + s) * kFlagStride;  // top's from_bottom[s]
       else
         f = p.bot_flags + (size_t)s * kFlagStride;                  // bottom's from_top[s]
-      if ((threadIdx.x & 31) == 0) st_release_sys(f, j < T ? k + j : k + T);
+      if ((threadIdx.x & 31) == 0) {
+        if (p.gpu_scope) st_release_gpu(f, j < T ? k + j : k + T);
+        else st_release_sys(f, j < T ? k + j : k + T);
+      }
     }
   }
 }
@@ -544,17 +577,32 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
   const bool rtop = top_blk && !deep_top, rbot = bot_blk && !deep_bot;
   double acc = 0.0;
   // round 1 before the march (all threads: the producer must not read halo rows before the wait)
+  UC_TRACE_AT(0);
+#if UC_TRACE
+  if (threadIdx.x == 0 && uc_trace_ptr) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    uc_trace_ptr[blockIdx.x * 16 + 14] = smid;
+  }
+#endif
   if (rtop) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, true, true, acc);
   if (rbot) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, 1, false, true, acc);
+  UC_TRACE_AT(1);
   const int a = deep_top ? lo : max(lo, PT + 1);
   const int b = deep_bot ? hi : min(hi, p.n - PT);
   if (a <= b) {
     // fixed columns (0, NX-1) among the block's lanes, ghosts included: keep them fixed
     const int xs4 = s * p.strip4;
-    const bool diri = xs4 <= 1 || xs4 + p.strip4 >= p.nx4 - 1;
+    // per WARP, not per block: only the warps whose lanes (ghosts included) hold column 0 or
+    // NX-1 need the select that keeps it fixed (2 FSEL per float4 per level); the other warps of
+    // the two edge strips run the plain march (the edge strips were the slowest blocks, trace
+    // in profiles/r2_trace_blocks.txt).  The producer warp's path is the same in both instances.
+    const int wx0 = xs4 + warp_id_uniform() * Ghost<G>::kOwn - G;  // float4 column of lane 0
+    const bool diri = (wx0 <= 0 && 0 < wx0 + 32) || (wx0 <= p.nx4 - 1 && p.nx4 - 1 < wx0 + 32);
     if (diri) march_t<T, NL, true, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
     else march_t<T, NL, false, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
   }
+  UC_TRACE_AT(2);
   if ((rtop || rbot) && (int)threadIdx.x < p.consumers) {
 #if UC_ROUNDS_NOINLINE
     acc += t_rounds_after<T, NL, G>(p, src, dst, par, s, k, rtop, rbot);
@@ -562,6 +610,7 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
     for (int j = 2; j <= T; ++j) {  // consumers only (named barrier 1)
       if (rtop) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, true, false, acc);
       if (rbot) t_round<T, NL>(p, src, dst, par ^ 1, s, g, k, j, false, false, acc);
+      UC_TRACE_AT(1 + j);
     }
 #endif
   }
@@ -633,6 +682,7 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
     __threadfence();
     finish_iteration(p, nl > 0, smem, T);
   }
+  UC_TRACE_AT(15);
 }
 
 }  // namespace uc

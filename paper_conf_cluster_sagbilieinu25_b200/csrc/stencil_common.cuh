@@ -146,12 +146,26 @@ __device__ __forceinline__ void wait_strip_flags(const JacobiParams& p, int base
 // provably warp-uniform, so the code after it stays provably converged (a single-thread spin
 // loop makes the compiler guard every later shuffle with a divergence check and every later
 // mbarrier wait with a reconvergence region -- ~10 % more instructions in the march).
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// gpu = true when every party of the protocol is on this GPU (.gpu scope suffices)
 __device__ __forceinline__ bool wait_ge_warp(const uint64_t* sig, uint64_t v, unsigned long long timeout_ns,
-                                             unsigned int* err) {
-  if (__all_sync(kFull, uc_dev_ld_acquire(sig) >= v)) return true;
+                                             unsigned int* err, bool gpu = false) {
+  if (__all_sync(kFull, (gpu ? ld_acquire_gpu(sig) : uc_dev_ld_acquire(sig)) >= v)) return true;
   const unsigned long long t0 = uc_dev_globaltimer();
   unsigned ns = 32;
-  while (!__all_sync(kFull, uc_dev_ld_relaxed(sig) >= v)) {
+  while (!__all_sync(kFull, (gpu ? ld_relaxed_gpu(sig) : uc_dev_ld_relaxed(sig)) >= v)) {
     const bool give_up = uc_dev_globaltimer() - t0 > timeout_ns || *(volatile unsigned int*)err;
     if (__any_sync(kFull, give_up)) {
       if ((threadIdx.x & 31) == 0) atomicOr(err, 1u);
@@ -160,13 +174,16 @@ __device__ __forceinline__ bool wait_ge_warp(const uint64_t* sig, uint64_t v, un
     __nanosleep(ns);
     if (ns < 256) ns <<= 1;
   }
-  asm volatile("fence.acq_rel.sys;" ::: "memory");  // the observing load + fence = acquire
+  // the observing relaxed load + fence = acquire
+  if (gpu) asm volatile("fence.acq_rel.gpu;" ::: "memory");
+  else asm volatile("fence.acq_rel.sys;" ::: "memory");
   return true;
 }
 __device__ __forceinline__ void wait_strip_flags_warp(const JacobiParams& p, int base, int s, uint64_t v) {
   const int s0 = s > 0 ? s - 1 : 0;
   const int s1 = s + 1 < p.strips ? s + 1 : s;
-  for (int j = s0; j <= s1; ++j) wait_ge_warp(p.my_flags + (size_t)(base + j) * kFlagStride, v, p.timeout_ns, p.err);
+  for (int j = s0; j <= s1; ++j)
+    wait_ge_warp(p.my_flags + (size_t)(base + j) * kFlagStride, v, p.timeout_ns, p.err, p.gpu_scope != 0);
 }
 // warp index, broadcast from lane 0: branches on it are known warp-uniform
 __device__ __forceinline__ int warp_id_uniform() { return __shfl_sync(kFull, (int)threadIdx.x >> 5, 0); }
