@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--mode", default="device", choices=["device", "host"])
-    ap.add_argument("--host-path", default="1,1",
+    ap.add_argument("--host-path", default="1,0",
                     help="host mode: deep_halo,overlap (uc_jacobi_set_host_path); 0,0 = the paper's Listing 1")
     ap.add_argument("--nx", type=int, default=NX)
     ap.add_argument("--ny-per-gpu", type=int, default=NY_PER_GPU)
@@ -59,6 +59,9 @@ def parse():
     ap.add_argument("--iters-per-step", type=int, default=ITERS_PER_STEP)
     ap.add_argument("--norm-every", type=int, default=NORM_EVERY)
     ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--inject-delay-us", type=float, default=0.0,
+                    help="MEASUREMENT ONLY: release every boundary-round flag this much later (NVLink-like "
+                         "latency on one GPU) to measure how much of it the launch hides")
     ap.add_argument("--same-device", action="store_true",
                     help="TEST ONLY: put every rank on cuda:0 (exercises the multi-process path on a 1-GPU box; "
                          "ranks time-slice the GPU, so the numbers are not a benchmark)")
@@ -67,7 +70,7 @@ def parse():
     ap.add_argument("--cpu-sample-iters", type=int, default=12)
     ap.add_argument("--variant", type=int, default=-1,
                     help="0 register march, 1 TMA-staged, 2 dynamic tiles, 3 persistent, 4 two iterations per "
-                         "launch, 5 T iterations per launch (T = --tile-rows; -1: library default = 5, T = 6)")
+                         "launch, 5 T iterations per launch (T = --tile-rows; -1: library default = 5, T = 8)")
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--block-x", type=int, default=0)
@@ -206,6 +209,8 @@ def run_ours(a):
     import numpy as np
     import torch
 
+    if a.inject_delay_us > 0:
+        os.environ["UC_INJECT_PUT_DELAY_NS"] = str(int(a.inject_delay_us * 1000))
     import paper_conf_cluster_sagbilieinu25_b200 as U
 
     rank, world, local = dist_env()
@@ -440,6 +445,7 @@ def run_ours(a):
                        else "configs[2] (strong, 16384^2 total)",
                        "nx": nx, "ny_global": ny, "rows_per_gpu": n, "iters_per_step": ips,
                        "norm_every": a.norm_every, "mode": a.mode, "cuda_graph": use_graph,
+                       "injected_flag_delay_us": a.inject_delay_us or None,
                        "host_path": ({"deep_halo": host_path[0], "overlap": host_path[1]} if a.mode == "host"
                                      else None),
                        "parallelism": f"y-slab x{world}", "l2": "inputs > L2 (2 slabs x "

@@ -222,6 +222,11 @@ __device__ __forceinline__ void t_round(const JacobiParams& p, const float* src,
 #if UC_ROUND_SYS_FENCE
       else __threadfence_system();
 #endif
+      if (p.put_delay_ns) {  // injected link latency (measurement knob): the flag arrives later
+        const unsigned long long t0 = __shfl_sync(kFull, globaltimer(), 0);
+        while (__shfl_sync(kFull, globaltimer(), 0) - t0 < p.put_delay_ns) {
+        }
+      }
       uint64_t* f;
       if (j < T)
         f = (top ? p.top_h1_flags : p.bot_h1_flags) + (size_t)(j - 1) * 2 * p.flag_half * kFlagStride +
@@ -300,9 +305,20 @@ __device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx
 #ifndef UC_HOIST_62
 #define UC_HOIST_62 3  // levels hoisted at <6, 2> (A/B: 0 / 2 / 3 / 4 -> 3509 / 3546 / 3568 / 3530 GLUPS)
 #endif
+#ifndef UC_HOIST_82
+#define UC_HOIST_82 2  // levels hoisted at <8, 2> (A/B, march alone: 0/2/3/4/8 -> 0.492/0.487/0.489/0.488/0.536 ms: hoisting all spills)
+#endif
+#ifndef UC_HOIST_72
+#define UC_HOIST_72 7  // levels hoisted at <7, 2> (A/B)
+#endif
 // levels whose neighbours are shuffled before the ring wait (the rest after it)
 template <int T, int G>
-constexpr int kHoistLevels = UC_HOIST_ALL == 1 ? T : UC_HOIST_ALL == -1 ? 0 : (T == 6 && G == 2) ? UC_HOIST_62 : T;
+constexpr int kHoistLevels = UC_HOIST_ALL == 1    ? T
+                             : UC_HOIST_ALL == -1 ? 0
+                             : (T == 6 && G == 2) ? UC_HOIST_62
+                             : (T == 7 && G == 2) ? UC_HOIST_72
+                             : (T == 8 && G == 2) ? UC_HOIST_82
+                                                  : T;
 
 // One row of the T-level march: fetch the next A_k row, advance every level, store.
 template <int T, int NL, bool DIRI, bool STORE, int HOIST>

@@ -73,6 +73,8 @@ struct JacobiParams {
   int deep_halo;                       // variant 5, host mode: T halo rows per side with a neighbour
   int part;                            // variant 5: 0 whole launch, 1 edge chunks, 2 other chunks
   int partial_base;                    // index of this launch's first block partial
+  unsigned put_delay_ns;               // test/measurement knob (UC_INJECT_PUT_DELAY_NS): each boundary
+                                       // round's flag is released this much later (NVLink-like latency)
   int gpu_scope;                       // 1: top and bottom live on this GPU (same process): halo
                                        // flags at .gpu scope instead of .sys
   double* partials;                    // local [grid] per-block partial sums

@@ -35,7 +35,9 @@ def main():
     # (self-exchange), P = 2 (top == bottom) and P = 3 (distinct peers); ne = 6 keeps every launch
     # at T = 6 (a norm cadence below T demotes launches)
     t6 = [dict(P=1, mode="device", variant=5, T=6, ne=6, iters=13), dict(P=2, mode="device", variant=5, T=6, ne=0, iters=12),
-          dict(P=3, mode="device", variant=5, T=6, ne=6, iters=12)]
+          dict(P=3, mode="device", variant=5, T=6, ne=6, iters=12),
+          dict(P=1, mode="device", variant=5, T=8, ne=8, iters=17), dict(P=2, mode="device", variant=5, T=8, ne=0, iters=16),
+          dict(P=3, mode="device", variant=5, T=8, ne=8, iters=16)]
     if os.environ.get("UC_SANITIZE_T6_ONLY"):
         cases = t6
     else:
@@ -51,10 +53,10 @@ def main():
                         variant=c["variant"], tile_rows=c.get("T", 0), use_graph=False)
         want, _ = oracle.jacobi_run(gen.global_field(nx, ny * P, "ring"), iters, "ring")
         assert_slabs_equal_global(res["final"], want, P, "ring")
-        if c["variant"] == 5 and c.get("T", 0) == 6:
+        if c["variant"] == 5 and c.get("T", 0) in (6, 8):
             import paper_conf_cluster_sagbilieinu25_b200 as U
-            plan = U.launch_plan(5, 6, 1, ny, iters, ne)
-            assert plan[:2] == [6, 6], plan
+            plan = U.launch_plan(5, c["T"], 1, ny, iters, ne)
+            assert plan[0] == c["T"], plan
         print("ok", c, flush=True)
     print("SANITIZE_RUN_DONE")
 

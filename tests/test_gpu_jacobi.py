@@ -267,14 +267,15 @@ def test_constant_field_fixed_and_zero_norm():
 def test_full_size_16384_single_gpu_bench_configuration():
     """BASELINE.json configs[2]/[3] at P = 1 (16384^2 fp32, 1 GiB per slab), in the launch
     configuration bench.py times (device mode, ring, CUDA graph, default geometry = variant 5,
-    six iterations per launch with two ghost lanes, 9-row ring): the whole grid bit-exact vs the
-    oracle after 12, 14 (a two-iteration launch at the end) and 17 iterations (a five-iteration
-    one), norms within 1e-5 on every level."""
-    res = _check(16384, 16384, 1, "ring", "device", 12, norm_every=6)
-    assert res["launch"]["variant"] == 5 and res["launch"]["stages"] == 9 and res["launch"]["tile_rows"] == 6
-    assert res["launch"]["block"] == 256
+    eight iterations per launch with two ghost lanes, 9-row ring): the whole grid bit-exact vs the
+    oracle after 16 (two launches of 8, a norm on each), 14 (a norm cadence of 7 demotes to 7)
+    and 25 iterations (8, 8, then the remainder split: 5, 4), norms within 1e-5 on every level."""
+    res = _check(16384, 16384, 1, "ring", "device", 16, norm_every=8)
+    assert res["launch"]["variant"] == 5 and res["launch"]["stages"] == 9 and res["launch"]["tile_rows"] == 8
+    assert res["launch"]["block"] == 256 and res["counts"][8] == 2
     _check(16384, 16384, 1, "ring", "device", 14, norm_every=7)
-    _check(16384, 16384, 1, "ring", "device", 17, norm_every=0)
+    res = _check(16384, 16384, 1, "ring", "device", 25, norm_every=0)
+    assert res["counts"][8] == 2 and res["counts"][5] == 1 and res["counts"][4] == 1
 
 
 def test_full_size_host_mode():

@@ -186,53 +186,69 @@ def test_config1_4096_2ranks_1000_iterations(T):
 
 
 # ---------------------------------------------------------------------------------------------
-# The shipped default, jacobi_t_kernel<6, 2>, where the multi-rank protocol can break: distinct
-# top and bottom peers (P >= 3), the chain ends, full-size geometry.  A norm cadence below T
-# demotes launches, so these runs use norm_every 0 or a multiple of 6 and assert (through the
-# device launch counters, uc_jacobi_launch_counts) that T = 6 launches really ran.
+# The deep instances -- the shipped default jacobi_t_kernel<8, 2> and <6, 2> -- where the
+# multi-rank protocol can break: distinct top and bottom peers (P >= 3), the chain ends, the
+# thinnest slabs, full-size geometry.  A norm cadence below T demotes launches, so these runs use
+# norm_every 0 or a multiple of T and assert (device launch counters, uc_jacobi_launch_counts)
+# that depth-T launches really ran; the harness also checks every launch against the plan.
+DEEP = [6, 8]
 
-@pytest.mark.parametrize("P", [3, 4, 8])
-@pytest.mark.parametrize("topology,ne", [("ring", 0), ("ring", 6), ("dirichlet", 12)])
-def test_t6_distinct_peers(P, topology, ne):
-    res = _check(1028, 24 * P, P, topology, "device", 18, norm_every=ne)  # library default: T = 6
-    assert res["launch"]["variant"] == 5 and res["launch"]["tile_rows"] == 6
+
+def _deep(res, T, n_expected):
+    assert res["launch"]["variant"] == 5 and res["launch"]["tile_rows"] == T
     for c in res["counts_all"]:
-        assert c[6] == 3 and sum(c) == 3, c
+        assert c[T] == n_expected, (T, c)
 
 
-@pytest.mark.parametrize("P,rows", [(3, 12), (4, 13), (2, 12)])
-def test_t6_thinnest_slabs(P, rows):
-    """n = 2T = 12 (every chunk is a boundary chunk) and n = 13 (ragged), wide enough for two
-    strips per rank."""
+@pytest.mark.parametrize("T", DEEP)
+@pytest.mark.parametrize("P", [3, 4, 8])
+@pytest.mark.parametrize("topology,nem", [("ring", 0), ("ring", 1), ("dirichlet", 2)])
+def test_deep_distinct_peers(T, P, topology, nem):
+    res = _check(1028, 4 * T * P, P, topology, "device", 3 * T, norm_every=nem * T, **_v5(T))
+    _deep(res, T, 3)
+
+
+@pytest.mark.parametrize("T", DEEP)
+@pytest.mark.parametrize("P,extra", [(3, 0), (4, 1), (2, 0)])
+def test_deep_thinnest_slabs(T, P, extra):
+    """n = 2T (every chunk is a boundary chunk) and n = 2T + 1 (ragged), two strips per rank."""
     for topology in ("ring", "dirichlet"):
-        res = _check(2052, rows * P, P, topology, "device", 12, norm_every=6)
-        assert all(c[6] == 2 for c in res["counts_all"]), res["counts_all"]
+        res = _check(2052, (2 * T + extra) * P, P, topology, "device", 2 * T, norm_every=T, **_v5(T))
+        _deep(res, T, 2)
 
 
-def test_t6_random_values_p3():
-    nx, ny = 1028, 72
-    rng = np.random.default_rng(6)
+@pytest.mark.parametrize("T", DEEP)
+def test_deep_random_values_p3(T):
+    nx, ny = 1028, 12 * T
+    rng = np.random.default_rng(T)
     init = rng.random((ny + 2, nx), dtype=np.float32)
     init[0], init[-1] = init[ny], init[1]
-    res = _check(nx, ny, 3, "ring", "device", 24, norm_every=6, init=init)
-    assert res["counts"][6] == 4
+    res = _check(nx, ny, 3, "ring", "device", 4 * T, norm_every=T, init=init, **_v5(T))
+    _deep(res, T, 4)
 
 
-def test_t6_config1_default():
+def test_default_is_t8_config1():
     """configs[1] (4096^2, 2 ranks, 1000 iterations, norm every 100) at the library default:
-    166 launches of T = 6 and one of T = 4."""
+    T = 8, 125 launches of 8."""
     res = _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100)
-    assert res["launch"]["tile_rows"] == 6
+    _deep(res, 8, 125)
+
+
+def test_t6_config1():
+    """configs[1] at T = 6: 165 launches of 6 and two of 5 (the remainder 4 split with the launch
+    before it)."""
+    res = _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, **_v5(6))
     for c in res["counts_all"]:
-        assert c[6] == 166 and c[4] == 1 and sum(c) == 167, c
+        assert c[6] == 165 and c[5] == 2 and sum(c) == 167, c
 
 
-def test_t6_config3_two_ranks():
+@pytest.mark.parametrize("T", DEEP)
+def test_deep_config3_two_ranks(T):
     """configs[3] at P = 2 (16384 x 32768 global, 16384^2 per rank: the bench's per-GPU geometry
-    with real neighbours), 13 iterations with a norm every 6: launches 6, 6, 1."""
-    res = _check(16384, 32768, 2, "ring", "device", 13, norm_every=6)
-    for c in res["counts_all"]:
-        assert c[6] == 2 and c[1] == 1, c
+    with real neighbours), 2T + 1 iterations with a norm every T: launches T, then the remainder
+    1 split with the launch before it."""
+    res = _check(16384, 32768, 2, "ring", "device", 2 * T + 1, norm_every=T, **_v5(T))
+    _deep(res, T, 1)
 
 
 def test_two_virtual_ranks_need_concurrent_kernels():
@@ -294,11 +310,20 @@ def test_two_virtual_ranks_need_concurrent_kernels():
 def test_host_paths(deep, overlap, topology, iters, ne):
     res = _check(1028, 192, 1, topology, "host", iters, norm_every=ne, host_path=(deep, overlap))
     if deep and ne in (0, 6):
-        assert res["counts"][6] >= 2, res["counts"]
+        assert res["counts"][6] >= 1, res["counts"]
 
 
 @pytest.mark.parametrize("deep,overlap", [(1, 0), (1, 1), (0, 1)])
 def test_host_paths_full_size(deep, overlap):
     res = _check(16384, 16384, 1, "ring", "host", 13, norm_every=6, host_path=(deep, overlap))
     if deep:
-        assert res["counts"][6] == 2 and res["counts"][1] == 1, res["counts"]
+        assert res["counts"][6] == 1 and res["counts"][4] == 1 and res["counts"][3] == 1, res["counts"]
+
+
+@pytest.mark.parametrize("P,topology", [(3, "ring"), (2, "dirichlet")])
+def test_t6_injected_flag_latency(monkeypatch, P, topology):
+    """Every boundary-round flag released 20 us late (UC_INJECT_PUT_DELAY_NS, the knob behind
+    bench.py --inject-delay-us): the waits absorb it, the grid stays bit-exact."""
+    monkeypatch.setenv("UC_INJECT_PUT_DELAY_NS", "20000")
+    res = _check(1028, 32 * P, P, topology, "device", 24, norm_every=8)
+    assert all(c[8] == 3 for c in res["counts_all"])

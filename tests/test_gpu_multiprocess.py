@@ -55,13 +55,18 @@ def test_multiprocess_ipc_device_mode(tmp_path, P, topology, mode):
 
 
 @pytest.mark.parametrize("P,topology", [(2, "ring"), (3, "ring"), (4, "ring"), (3, "dirichlet")])
-def test_multiprocess_ipc_t6(tmp_path, P, topology):
-    """The shipped jacobi_t_kernel<6, 2> across PROCESSES (CUDA IPC peers): 20 iterations with a
-    norm every 6 are launches 6, 6, 6, 2 on every rank (device counters)."""
-    res = _run(tmp_path, P, 1028, 16 * P, 20, 6, topology, "device")
+def test_multiprocess_ipc_deep(tmp_path, P, topology):
+    """The shipped jacobi_t_kernel<8, 2> across PROCESSES (CUDA IPC peers): 24 iterations with a
+    norm every 8 are three launches of 8 on every rank (device counters); with a norm every 6 the
+    launches demote to <6, 2>: 6, 6, 6, 6."""
+    res = _run(tmp_path, P, 1028, 16 * P, 24, 8, topology, "device")
     for x in res:
         c = list(x["counts"])
-        assert c[6] == 3 and c[2] == 1 and sum(c) == 4, c
+        assert c[8] == 3 and sum(c) == 3, c
+    res = _run(tmp_path, P, 1028, 16 * P, 24, 6, topology, "device")
+    for x in res:
+        c = list(x["counts"])
+        assert c[6] == 4 and sum(c) == 4, c
 
 
 # ---- one GPU per rank (NCCL allows one rank per GPU): run where the box has >= 2 GPUs
@@ -88,7 +93,7 @@ def test_host_paths_multi_gpu(tmp_path, deep, overlap, P, topology):
     res = _run(tmp_path, P, 2052, 96 * P, 25, 6, topology, "host", same_device=False, host_path=(deep, overlap))
     if deep:
         for x in res:
-            assert list(x["counts"])[6] == 4, list(x["counts"])
+            assert list(x["counts"])[6] == 3, list(x["counts"])
 
 
 @pytest.mark.skipif("_gpus() < 4", reason="needs >= 4 GPUs")

@@ -21,6 +21,9 @@ def restated(variant, levels, mode, n, iters, ne):
                 t -= 1
             plan.append(t)
             i += t
+        if len(plan) >= 2 and plan[-1] < plan[-2] - 1:  # even split of a short remainder
+            tot = plan[-2] + plan[-1]
+            plan[-2:] = [(tot + 1) // 2, tot // 2]
         return plan
     if variant == 4 and mode == DEV and n >= 2 and ne != 1:
         return [2] * (iters // 2) + [1] * (iters % 2)
@@ -48,21 +51,30 @@ def test_plan_rules(variant, levels, mode, n):
                     for k0 in range(0, 2 * max(ne, 1) + 1):
                         norms = sum(1 for kk in range(k0, k0 + t) if ne > 0 and kk % ne == 0)
                         assert norms <= 1
-            # greedy: only the last launch of a run may be shorter than the deepest feasible one
+            # greedy: only the last two launches of a run may be shorter than the deepest feasible
+            # one, and they differ by at most 1 after the split of a short remainder
             if variant == 5 and plan:
-                assert all(t == plan[0] for t in plan[:-1]) and plan[-1] <= plan[0]
+                assert all(t == plan[0] for t in plan[:-2]) and all(t <= plan[0] for t in plan)
+                if len(plan) >= 2:
+                    assert plan[-1] >= plan[-2] - 1
 
 
 def test_bench_configuration_plan():
     """The default bench step: 100 iterations, norm every 100, 16384 rows -> 25 launches of 4."""
     assert U.launch_plan(5, 4, DEV, 16384, 100, 100) == [4] * 25
     assert U.launch_plan(5, 4, DEV, 2048, 100, 100) == [4] * 25    # configs[2] slab at P = 8
-    assert U.launch_plan(5, 4, DEV, 6, 10, 0) == [3, 3, 3, 1]       # n = 6: T' = 3
-    assert U.launch_plan(5, 4, DEV, 16384, 10, 3) == [3, 3, 3, 1]   # norm every 3 < T
+    assert U.launch_plan(5, 4, DEV, 6, 10, 0) == [3, 3, 2, 2]       # n = 6: T' = 3 (3 + 1 split)
+    assert U.launch_plan(5, 4, DEV, 16384, 10, 3) == [3, 3, 2, 2]   # norm every 3 < T
     assert U.launch_plan(5, 4, HOST, 16384, 3, 0) == [1, 1, 1]
-    assert U.launch_plan(4, 0, DEV, 16384, 5, 0) == [2, 2, 1]
-    # two ghost lanes (T up to 8): 100 = 12 x 8 + 4
-    assert U.launch_plan(5, 8, DEV, 16384, 100, 100) == [8] * 12 + [4]
+    assert U.launch_plan(4, 0, DEV, 16384, 5, 0) == [2, 2, 1]      # variant 4: pairs + 1
+    # two ghost lanes (T up to 8): 100 = 11 x 8 + 6 + 6 (the short remainder 4 is split evenly)
+    assert U.launch_plan(5, 8, DEV, 16384, 100, 100) == [8] * 11 + [6, 6]
+    assert U.launch_plan(5, 6, DEV, 16384, 100, 100) == [6] * 15 + [5, 5]
+    assert U.launch_plan(5, 8, DEV, 16384, 9, 0) == [5, 4]
+    # deep-halo host mode follows the device plan; the paper's host path is one per launch
+    assert U.launch_plan(5, 6, HOST | U.UC_PLAN_DEEP_HALO, 16384, 13, 6) == [6, 4, 3]
+    assert U.launch_plan(5, 6, DEV, 16384, 1000, 100) == [6] * 165 + [5, 5]  # configs[1]
+    assert U.launch_plan(5, 6, HOST, 16384, 3, 0) == [1, 1, 1]
     assert U.launch_plan(5, 8, DEV, 10, 100, 0) == [5] * 20           # n = 10: T' = 5
 
 
