@@ -164,6 +164,13 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.lines.append((time.time(), line.strip()))
 
+    def wait_ready(self, timeout=5.0):
+        """nvidia-smi needs a few hundred ms before its first sample; a short timed region that
+        starts earlier records no clocks at all."""
+        t = time.time()
+        while self.proc is not None and not self.lines and time.time() - t < timeout:
+            time.sleep(0.02)
+
     def mark_start(self):
         """Started before the warm-up (nvidia-smi needs ~0.1-0.3 s to start); the timed region is
         [mark_start, mark_stop] and only samples that arrive inside it count."""
@@ -248,6 +255,7 @@ def run_ours(a):
     for _ in range(a.warmup):
         step()
     coord.sync()
+    clocks.wait_ready()
     counts0 = J.launch_counts()
 
     # ---------------- timed region: K steps, events on the coordinator's stream
@@ -529,8 +537,9 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
         co.signal_wait(row, nx * 4, nx * 4, sig, 16, i, comm.top)
     x1.record(st2)
     co.sync()
-    # a two-iteration launch exchanges two rounds of boundary rows
-    t_x = x0.elapsed_time(x1) / reps * per_launch
+    # a launch of T iterations exchanges T rounds of boundary rows; under injected flag latency
+    # (--inject-delay-us) every round of the exchange alone costs that much more
+    t_x = x0.elapsed_time(x1) / reps * per_launch + per_launch * a.inject_delay_us / 1e3
     comm.barrier()
     row.free()
     sig.free()
@@ -543,7 +552,8 @@ def halo_overlap(a, U, torch, dist, env, rank, world, local, nx, n, mode, k_full
     return {"hidden_fraction": None if hidden is None else round(hidden, 4), "t_full_ms": round(t_full, 5),
             "t_compute_ms": round(t_comp, 5), "t_xchg_ms": round(t_x, 5),
             "note": f"per launch ({per_launch} iteration(s)); t_xchg = standalone put_signal of both boundary "
-                    f"rows + waits, x{per_launch} rounds"}
+                    f"rows + waits, x{per_launch} rounds" + (f", + {a.inject_delay_us} us injected flag latency per "
+                                                             "round" if a.inject_delay_us else "")}
 
 
 def cpu_baseline(nx, ny, iters, norm_every):

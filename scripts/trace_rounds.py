@@ -3,8 +3,8 @@
     python paper_conf_cluster_sagbilieinu25_b200/build.py --define UC_TRACE=1 --out build/ab/lib_trace.so
     UC_LIB_PATH=build/ab/lib_trace.so python scripts/trace_rounds.py [--ny 16384] [--shrink S]
 
-%globaltimer stamps (ns) per block: 0 start, 1 after round 1, 2 after the march, 3..7 after rounds
-2..6, 15 end.  Prints the launch span and, for interior and edge (boundary-round) blocks, the
+%globaltimer stamps (ns) per block: 0 start, 1 after round 1, 2 after the march, 1+j after round j
+(j = 2..T), 14 the SM id, 15 end.  Prints the launch span and, for interior and edge (boundary-round) blocks, the
 phase durations relative to the launch start."""
 import argparse
 import ctypes as C
@@ -33,8 +33,9 @@ def main():
     co = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
     J = U.Jacobi(comm, a.nx, a.ny)
     info = J.launch_info()
+    T = info["tile_rows"]
     for _ in range(4):
-        J.run(co, 12, 0, use_graph=False)
+        J.run(co, 2 * T, 0, use_graph=False)
     co.sync()
     U.lib.uc_debug_trace_buffer.restype = C.c_void_p
     ptr = U.lib.uc_debug_trace_buffer()
@@ -53,7 +54,7 @@ def main():
     e = t[edge]
     print(f"edge blocks ({e.shape[0]}): round 1 done +{us(np.median(e[:,1]-t0)):.1f}, march end +{us(np.median(e[:,2]-t0)):.1f} "
           f"(max {us(np.max(e[:,2]-t0)):.1f})")
-    for j in range(2, 7):
+    for j in range(2, T + 1):
         d = e[:, 1 + j] - e[:, j]
         print(f"  round {j}: median {us(np.median(d)):.1f} us, max {us(np.max(d)):.1f}; done +{us(np.median(e[:,1+j]-t0)):.1f} "
               f"(max {us(np.max(e[:,1+j]-t0)):.1f})")
