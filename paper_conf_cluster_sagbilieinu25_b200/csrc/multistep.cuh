@@ -332,58 +332,6 @@ __device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64
   t_levels<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, L, R, out, pitch, acc);
 }
 
-#ifndef UC_SKEW
-#define UC_SKEW 0  // A/B knob: S > 0 = skewed level schedule in groups of S levels, 0 = fully chained
-#endif
-constexpr int kSkew = UC_SKEW > 0 ? UC_SKEW : 1;
-
-// Skewed schedule: the levels form groups of S = UC_SKEW; the first level of a group (j > 0,
-// j % S == 0) takes the previous group's row from the PREVIOUS step (pend[j-1]), so the groups of
-// one step are independent chains (T/S-way ILP) for D = (T-1)/S more float4 registers.  Level j+1
-// emits row r - j - 1 - j/S at step i (r = a - T + i); the A_{k+T} row a comes out at i = 2T + D
-// and the march runs D drain steps past the last ring row.  Same operations on the same operands
-// as t_levels: bit-identical results.
-template <int T, int NL, bool DIRI, bool STORE>
-__device__ __forceinline__ void t_levels_skew(float4 nv, const GhostLayout& g, int nx4, int a, int b, int i,
-                                              float4 (&w0)[T], float4 (&w1)[T], float4 (&pend)[T],
-                                              const float (&L)[T], const float (&R)[T], float*& out, size_t pitch,
-                                              double& acc) {
-  constexpr int S = kSkew;
-  float4 chain = nv, newp[T];
-#pragma unroll
-  for (int j = 0; j < T; ++j) {
-    const float4 in = (j > 0 && j % S == 0) ? pend[j - 1] : chain;
-    const float4 o = row_update_lr<DIRI>(w0[j], w1[j], in, L[j], R[j], g.x4, nx4);  // level j+1
-    if (NL == j + 1 && g.own) {
-      const int y = a - T + i - j - 1 - j / S;
-      if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
-    }
-    w0[j] = w1[j];
-    w1[j] = in;
-    if (j + 1 < T && (j + 1) % S == 0) newp[j] = o;
-    chain = o;
-  }
-#pragma unroll
-  for (int j = 0; j + 1 < T; ++j)
-    if ((j + 1) % S == 0) pend[j] = newp[j];
-  if (STORE) {
-    if (g.own) st4(out, chain);
-    out += pitch;
-  }
-}
-
-template <int T, int NL, bool DIRI, bool STORE, bool FETCH, int HOIST>
-__device__ __forceinline__ void t_step_skew(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
-                                            const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
-                                            float4 (&w0)[T], float4 (&w1)[T], float4 (&pend)[T], float*& out,
-                                            size_t pitch, double& acc) {
-  float L[T], R[T];
-  t_neighbours<T, 0, HOIST>(w1, L, R);
-  const float4 nv = FETCH ? t_fetch(ring, full, empty, ST, NS, g, cur) : make_float4(0.f, 0.f, 0.f, 0.f);
-  t_neighbours<T, HOIST, T>(w1, L, R);
-  t_levels_skew<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, pend, L, R, out, pitch, acc);
-}
-
 // Grouped march (UC_MARCH_GROUPED, the product build): the steady-state row loop runs in groups
 // of kGroup rows = kGroup ring stages, so every stage index, mbarrier address and ring offset of
 // the group is a compile-time constant (one ring phase flip per group instead of per-row stage
@@ -494,33 +442,6 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
   for (int j = 0; j < T; ++j) w0[j] = w1[j] = make_float4(0.f, 0.f, 0.f, 0.f);
   RingCursor cur{0, 0u};
   float* out = dst + (size_t)a * pitch + 4 * (size_t)g.x4;  // the A_{k+T} row a comes out at i = 2T
-#if UC_SKEW
-  if constexpr (T > 1 && (T - 1) / kSkew > 0) {
-    constexpr int D = (T - 1) / kSkew;  // skew delays along the level chain
-    constexpr int FILL = 2 * T + D;      // steps before the first A_{k+T} row (a) comes out
-    constexpr int H = kHoistLevels<T, G>;
-    float4 pend[T];
-#pragma unroll
-    for (int j = 0; j < T; ++j) pend[j] = make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll
-    for (int i = 0; i < FILL; ++i) {
-      if (i < rows)
-        t_step_skew<T, NL, DIRI, false, true, H>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, pend, out,
-                                                 pitch, acc);
-      else
-        t_step_skew<T, NL, DIRI, false, false, H>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, pend, out,
-                                                  pitch, acc);
-    }
-#pragma unroll(kTUnroll)
-    for (int i = FILL; i < rows; ++i)
-      t_step_skew<T, NL, DIRI, true, true, H>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, pend, out,
-                                              pitch, acc);
-    for (int i = max(rows, FILL); i < rows + D; ++i)  // drain: no ring row left
-      t_step_skew<T, NL, DIRI, true, false, H>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, pend, out,
-                                               pitch, acc);
-    return;
-  }
-#endif
   // the first 2T rows only fill the levels (rows >= 2T + 1 since a <= b)
 #pragma unroll
   for (int i = 0; i < 2 * T; ++i)

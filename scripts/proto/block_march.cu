@@ -54,7 +54,8 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
 #endif
   if (a <= b) {
     const int xs4 = s * p.strip4;
-    const bool diri = xs4 <= 1 || xs4 + p.strip4 >= p.nx4 - 1;
+    const int wx0 = xs4 + warp_id_uniform() * Ghost<G>::kOwn - G;
+    const bool diri = (wx0 <= 0 && 0 < wx0 + 32) || (wx0 <= p.nx4 - 1 && p.nx4 - 1 < wx0 + 32);
     if (diri) march_t<T, 0, true, G>(p, p.slab[0], p.slab[1], s, g, a, b, acc, ring, full, empty, false);
     else march_t<T, 0, false, G>(p, p.slab[0], p.slab[1], s, g, a, b, acc, ring, full, empty, false);
   }
@@ -102,7 +103,8 @@ int main(int argc, char** argv) {
   auto kern = proto_kernel<PROTO_T, PROTO_G>;
   CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int bps = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kern, nc + 32, smem));
+  const int XT = 32;  // the producer warp
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kern, nc + XT, smem));
   cudaFuncAttributes fa;
   CK(cudaFuncGetAttributes(&fa, kern));
   if (chunks <= 0) chunks = (148 * bps) / strips;
@@ -159,9 +161,9 @@ int main(int argc, char** argv) {
   auto fk = jacobi_t_kernel<PROTO_T, PROTO_G>;
   CK(cudaFuncSetAttribute(fk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   CK(cudaFuncGetAttributes(&fa, fk));
-#define KLAUNCH fk<<<grid, nc + 32, smem>>>(p)
+#define KLAUNCH fk<<<grid, nc + XT, smem>>>(p)
 #else
-#define KLAUNCH kern<<<grid, nc + 32, smem>>>(p)
+#define KLAUNCH kern<<<grid, nc + XT, smem>>>(p)
 #endif
   KLAUNCH;
   CK(cudaGetLastError());
