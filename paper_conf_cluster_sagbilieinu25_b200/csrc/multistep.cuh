@@ -113,6 +113,115 @@ __device__ __forceinline__ float4 row_update_g(float4 up, float4 c, float4 dn, i
   return row_update_lr<DIRI>(up, c, dn, L, R, x4, nx4);
 }
 
+// ---- the march's register frame
+// A row's four columns x0..x3 live in two 64-bit register pairs, P = (x0, x3) and Q = (x1, x2),
+// instead of (x0, x1) | (x2, x3).  Then both horizontal sums of a level are single packed adds on
+// pairs as they stand: (h0, h3) = (L, R) + Q, with the two shuffled neighbours landing in one
+// pair, and (h1, h2) = P + swap(Q), the swap being a free FADD2 operand modifier (.LO_HI).  A
+// level is 8 packed FP32 instructions + 2 shuffles (row_update_lr: 4 FADD + 6 packed + 2
+// shuffles).  Every value is the same IEEE operation on the same two operands as in
+// row_update_lr (addition commutes exactly): bit-identical.  The pairs are 64-bit values in the
+// source, so the register allocator keeps them as aligned pairs (with float4 rows it kept the
+// natural order and rebuilt the pairs at every use).  A row is permuted into the frame once as it
+// leaves the ring; the last level is computed straight into the natural order for the store.
+using pair_t = unsigned long long;
+struct Row2 {
+  pair_t p, q;  // (x0, x3), (x1, x2): f32x2 (lo, hi)
+};
+__device__ __forceinline__ pair_t pk2(float lo, float hi) {
+  pair_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+__device__ __forceinline__ void upk2(pair_t v, float& lo, float& hi) {
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
+}
+__device__ __forceinline__ pair_t f2add(pair_t a, pair_t b) {
+  pair_t r;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ pair_t f2add_swapped(pair_t a, pair_t b) {  // a + (b.hi, b.lo)
+  pair_t r;
+  asm("{\n .reg .b32 lo, hi;\n .reg .b64 s;\n mov.b64 {lo, hi}, %2;\n mov.b64 s, {hi, lo};\n"
+      " add.rn.f32x2 %0, %1, s;\n}"
+      : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ pair_t f2quarter(pair_t a) {
+  pair_t r;
+  asm("{\n .reg .b64 q;\n mov.b64 q, {%2, %2};\n mul.rn.f32x2 %0, %1, q;\n}" : "=l"(r) : "l"(a), "f"(0.25f));
+  return r;
+}
+__device__ __forceinline__ Row2 to_row2(float4 n) { return Row2{pk2(n.x, n.w), pk2(n.y, n.z)}; }
+// A ring row into the frame.  An LDS.128 lands in natural order, and a permutation by register
+// moves is a copy the allocator rematerialises at every use of the row (~14 moves per row of the
+// march); four exact scalar adds of -0 (x + -0 = x for every non-NaN x, -0 and subnormals
+// included) make the permuted pairs values of their own, one instruction per column.  The warps
+// that hold a fixed column (DIRI) copy, so a NaN payload in a Dirichlet column passes unchanged.
+#ifndef UC_PQ_ADD_PERMUTE
+#define UC_PQ_ADD_PERMUTE 1
+#endif
+template <bool DIRI>
+__device__ __forceinline__ Row2 ring_row2(float4 n) {
+  if (UC_PQ_ADD_PERMUTE && !DIRI)
+    return Row2{pk2(__fadd_rn(n.x, -0.f), __fadd_rn(n.w, -0.f)), pk2(__fadd_rn(n.y, -0.f), __fadd_rn(n.z, -0.f))};
+  return to_row2(n);
+}
+__device__ __forceinline__ float4 from_row2(Row2 r) {
+  float4 n;
+  upk2(r.p, n.x, n.w);
+  upk2(r.q, n.y, n.z);
+  return n;
+}
+// the horizontal neighbours (L, R) of a row as one pair: x3 of the lane on the left, x0 of the
+// lane on the right (lanes 0 / 31: their own values -- ghost lanes, discarded)
+__device__ __forceinline__ pair_t row2_lr(const Row2& c) {
+  float x0, x3;
+  upk2(c.p, x0, x3);
+  return pk2(__shfl_up_sync(kFull, x3, 1), __shfl_down_sync(kFull, x0, 1));
+}
+// new = 0.25f*((l+r)+(t+b)) for the 4 columns, in the frame
+template <bool DIRI, bool SC = false>
+__device__ __forceinline__ Row2 row2_update(const Row2& up, const Row2& c, const Row2& dn, pair_t lr, int x4, int nx4) {
+  static_assert(!(DIRI && SC), "fixed columns are not scaled");
+  const pair_t hp = f2add(lr, c.q);          // (L + x1, R + x2)  = (h0, h3)
+  const pair_t hq = f2add_swapped(c.p, c.q); // (x0 + x2, x3 + x1) = (h1, h2)
+  const pair_t vp = f2add(up.p, dn.p), vq = f2add(up.q, dn.q);
+  // SC (the scaled march, below): the level's sums themselves, 4x the level's values
+  Row2 o{SC ? f2add(hp, vp) : f2quarter(f2add(hp, vp)), SC ? f2add(hq, vq) : f2quarter(f2add(hq, vq))};
+  if (DIRI) {  // fixed columns 0 (x0) and NX-1 (x3), both in P
+    float a0, a3, c0, c3;
+    upk2(o.p, a0, a3);
+    upk2(c.p, c0, c3);
+    o.p = pk2(x4 == 0 ? c0 : a0, x4 == nx4 - 1 ? c3 : a3);
+  }
+  return o;
+}
+// the same level with the products as scalar multiplies written in natural column order (the
+// last level of the march: its row is only stored)
+template <bool DIRI, bool SC = false, int T = 1>
+__device__ __forceinline__ float4 row2_update_natural(const Row2& up, const Row2& c, const Row2& dn, pair_t lr, int x4,
+                                                      int nx4) {
+  static_assert(!(DIRI && SC), "fixed columns are not scaled");
+  const pair_t hp = f2add(lr, c.q);
+  const pair_t hq = f2add_swapped(c.p, c.q);
+  const pair_t vp = f2add(up.p, dn.p), vq = f2add(up.q, dn.q);
+  float s0, s3, s1, s2;
+  upk2(f2add(hp, vp), s0, s3);
+  upk2(f2add(hq, vq), s1, s2);
+  // SC: the sums are 4^(T-1) x the unscaled level's sums; 4^-T undoes the scale and the 0.25
+  constexpr float m = SC ? 1.0f / (float)(1u << (2 * T)) : 0.25f;
+  float4 o = make_float4(__fmul_rn(s0, m), __fmul_rn(s1, m), __fmul_rn(s2, m), __fmul_rn(s3, m));
+  if (DIRI) {
+    float c0, c3;
+    upk2(c.p, c0, c3);
+    o.x = x4 == 0 ? c0 : o.x;
+    o.w = x4 == nx4 - 1 ? c3 : o.w;
+  }
+  return o;
+}
+
 struct GhostLayout {
   int x4;        // float4 column of this thread (ghost lanes: the neighbour's edge column)
   bool in_grid;  // 0 <= x4 < nx4 (may be loaded)
@@ -261,39 +370,7 @@ __device__ __forceinline__ float4 t_fetch(const float* ring, uint64_t* full, uin
   return nv;
 }
 
-// Advance every level by the A_k row nv (the i-th row of the march) and store the A_{k+T} row
-// (STORE: from the 2T-th row on).
-// The horizontal neighbours of every level's middle row (w1[j], known before the step's new row
-// arrives): shuffled up front, off the level chain (new row -> level 1 -> ... -> level T).
-template <int T, int J0 = 0, int J1 = T>
-__device__ __forceinline__ void t_neighbours(const float4 (&w1)[T], float (&L)[T], float (&R)[T]) {
-#pragma unroll
-  for (int j = J0; j < J1; ++j) {
-    L[j] = __shfl_up_sync(kFull, w1[j].w, 1);    // lane 0: its own value (ghost lane, discarded)
-    R[j] = __shfl_down_sync(kFull, w1[j].x, 1);  // lane 31: likewise
-  }
-}
 
-template <int T, int NL, bool DIRI, bool STORE>
-__device__ __forceinline__ void t_levels(float4 nv, const GhostLayout& g, int nx4, int a, int b, int i,
-                                         float4 (&w0)[T], float4 (&w1)[T], const float (&L)[T], const float (&R)[T],
-                                         float*& out, size_t pitch, double& acc) {
-#pragma unroll
-  for (int j = 0; j < T; ++j) {
-    const float4 o = row_update_lr<DIRI>(w0[j], w1[j], nv, L[j], R[j], g.x4, nx4);  // level j+1, row r-j-1
-    if (NL == j + 1 && g.own) {
-      const int y = a - T + i - j - 1;
-      if (y >= a && y <= b) acc_sq(acc, o, w1[j]);
-    }
-    w0[j] = w1[j];
-    w1[j] = nv;
-    nv = o;
-  }
-  if (STORE) {
-    if (g.own) st4(out, nv);
-    out += pitch;
-  }
-}
 
 // Shuffle the neighbours of the next step's first HOIST levels before its ring wait, the rest
 // after it.  Measured per instance (profiles/r1_t8_sweep.txt, passes 7, 9): hoisting every level
@@ -320,17 +397,6 @@ constexpr int kHoistLevels = UC_HOIST_ALL == 1    ? T
                              : (T == 8 && G == 2) ? UC_HOIST_82
                                                   : T;
 
-// One row of the T-level march: fetch the next A_k row, advance every level, store.
-template <int T, int NL, bool DIRI, bool STORE, int HOIST>
-__device__ __forceinline__ void t_step(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
-                                       const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
-                                       float4 (&w0)[T], float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
-  float L[T], R[T];
-  t_neighbours<T, 0, HOIST>(w1, L, R);  // overlaps the ring wait and the shared-memory load
-  const float4 nv = t_fetch(ring, full, empty, ST, NS, g, cur);
-  t_neighbours<T, HOIST, T>(w1, L, R);
-  t_levels<T, NL, DIRI, STORE>(nv, g, nx4, a, b, i, w0, w1, L, R, out, pitch, acc);
-}
 
 // Grouped march (UC_MARCH_GROUPED, the product build): the steady-state row loop runs in groups
 // of kGroup rows = kGroup ring stages, so every stage index, mbarrier address and ring offset of
@@ -355,40 +421,134 @@ static_assert(kGroup % 3 == 0, "the group must be a multiple of the rotation per
 template <int G>
 constexpr int kStageFloats = 4 * (G == 1 ? kMaxBlock : kMaxBlockG2) + 2 * Ghost<G>::kPadG;
 
+
+// ---- the scaled march (UC_SCALED_MARCH, the product build; norm-free launches, warps without a
+// fixed column).  The 0.25 product of levels 1..T-1 is a quarter of the FP32 work of a level.  It is
+// dropped: level j keeps W_j = 4^j A_{k+j} (its plain sums (l+r)+(t+b) of level j-1's W), and the
+// last level multiplies by 4^-T.  Binary floating point rounds scale-invariantly by powers of two
+// as long as no value is subnormal or overflows, so then every W_j is exactly 4^j times the
+// unscaled iterate and A_{k+T} comes out bit-identical.  When is nothing subnormal?  If every
+// nonzero |A_k| value the warp reads is >= 2^(e) with e = -103 + 2T, all of them are integer
+// multiples of q = 2^(e-23) = 2^(-126+2T); sums and their roundings of multiples of q are again
+// multiples of q (a rounded result is a multiple of its own ulp, and ulp >= q or the sum is exact),
+// so a nonzero level-j value of the unscaled iteration is a multiple of q 4^-j >= 2^-126: normal,
+// and so is every scaled one (larger by 4^j).  Overflow: |W_j| <= 4^j max|A_k| (Jacobi averages),
+// so max|A_k| < 2^110 keeps 4^T max|A_k| far below 2^128 for T <= 8.  Each warp tracks the range
+// of the A_k rows it takes from the ring (max |x|; min over nonzero |x| as an unsigned min of
+// (bits << 1) - 1, zero wrapping to the top); inf is out of range; a NaN propagates as the same
+// canonical NaN in both forms.  If any warp of a block saw a value out of range, the whole block
+// re-runs its march unscaled (the ring continues; A_k is untouched and the march's rows of A_{k+T}
+// are rewritten) -- the answer is always the unscaled iteration's.
+#ifndef UC_SCALED_MARCH
+#define UC_SCALED_MARCH 1
+#endif
+struct RowRange {
+  float amax;     // max |x|
+  unsigned wmin;  // min ((bits << 1) - 1): nonzero |x|'s biased exponent in the top byte, zero -> ~0
+};
+__device__ __forceinline__ void range_add(RowRange& r, float4 n) {
+  r.amax = fmaxf(fmaxf(r.amax, fabsf(n.x)), fmaxf(fmaxf(fabsf(n.y), fabsf(n.z)), fabsf(n.w)));
+  const unsigned w0 = (__float_as_uint(n.x) << 1) - 1u, w1 = (__float_as_uint(n.y) << 1) - 1u;
+  const unsigned w2 = (__float_as_uint(n.z) << 1) - 1u, w3 = (__float_as_uint(n.w) << 1) - 1u;
+  r.wmin = min(min(r.wmin, w0), min(min(w1, w2), w3));
+}
+template <int T>
+__device__ __forceinline__ bool range_ok(const RowRange& r) {
+  constexpr unsigned kMinBiasedExp = 24 + 2 * T;  // 2^(-103+2T)
+  return r.amax < 0x1p110f && r.wmin >= (kMinBiasedExp << 24) - 1u;
+}
+
+// One row of the T-level march: fetch the next A_k row, advance every level, store the A_{k+T}
+// row (STORE: from the 2T-th row on).  The horizontal neighbours of every level's middle row
+// (w1[j], known before the step's new row arrives) are shuffled up front, off the level chain
+// (new row -> level 1 -> ... -> level T); the first HOIST levels' before the ring wait.
+template <int T, int J0, int J1>
+__device__ __forceinline__ void t_neighbours2(const Row2 (&w1)[T], pair_t (&lr)[T]) {
+#pragma unroll
+  for (int j = J0; j < J1; ++j) lr[j] = row2_lr(w1[j]);
+}
+template <int T, int NL, bool DIRI, bool STORE, bool SC>
+__device__ __forceinline__ void t_levels2(const Row2& n0, const GhostLayout& g, int nx4, int a, int b, int i,
+                                          Row2 (&w0)[T], Row2 (&w1)[T], const pair_t (&lr)[T], float*& out,
+                                          size_t pitch, double& acc) {
+  static_assert(!(SC && NL != 0), "norm launches run unscaled");
+  Row2 nv = n0;
+#pragma unroll
+  for (int j = 0; j < T - 1; ++j) {
+    const Row2 o = row2_update<DIRI, SC>(w0[j], w1[j], nv, lr[j], g.x4, nx4);  // level j+1, row r-j-1
+    if (NL == j + 1 && g.own) {
+      const int y = a - T + i - j - 1;
+      if (y >= a && y <= b) acc_sq(acc, from_row2(o), from_row2(w1[j]));
+    }
+    w0[j] = w1[j];
+    w1[j] = nv;
+    nv = o;
+  }
+  // level T (natural column order: only stored)
+  const float4 o = row2_update_natural<DIRI, SC, T>(w0[T - 1], w1[T - 1], nv, lr[T - 1], g.x4, nx4);
+  if (NL == T && g.own) {
+    const int y = a + i - 2 * T;  // a - T + i - j - 1 at j = T - 1
+    if (y >= a && y <= b) acc_sq(acc, o, from_row2(w1[T - 1]));
+  }
+  w0[T - 1] = w1[T - 1];
+  w1[T - 1] = nv;
+  if (STORE) {
+    if (g.own) st4(out, o);
+    out += pitch;
+  }
+}
+template <int T, int NL, bool DIRI, bool STORE, int HOIST, bool SC>
+__device__ __forceinline__ void t_step2(const float* ring, uint64_t* full, uint64_t* empty, int ST, int NS,
+                                        const GhostLayout& g, int nx4, int a, int b, int i, RingCursor& cur,
+                                        Row2 (&w0)[T], Row2 (&w1)[T], float*& out, size_t pitch, double& acc,
+                                        RowRange& rng) {
+  pair_t lr[T];
+  t_neighbours2<T, 0, HOIST>(w1, lr);
+  const float4 n = t_fetch(ring, full, empty, ST, NS, g, cur);
+  if (SC) range_add(rng, n);
+  const Row2 nv = ring_row2<DIRI>(n);
+  t_neighbours2<T, HOIST, T>(w1, lr);
+  t_levels2<T, NL, DIRI, STORE, SC>(nv, g, nx4, a, b, i, w0, w1, lr, out, pitch, acc);
+}
 // One group of kGroup rows starting at ring stage gbase (a multiple of kGroup), phase ph.
-template <int T, int NL, bool DIRI, int G, int HOIST>
-__device__ __forceinline__ void t_group(const float* ringp, uint64_t* full, uint64_t* empty, unsigned ph,
-                                        const GhostLayout& g, int nx4, int a, int b, int i0, float4 (&w0)[T],
-                                        float4 (&w1)[T], float*& out, size_t pitch, double& acc) {
+template <int T, int NL, bool DIRI, int G, int HOIST, bool SC>
+__device__ __forceinline__ void t_group2(const float* ringp, uint64_t* full, uint64_t* empty, unsigned ph,
+                                         const GhostLayout& g, int nx4, int a, int b, int i0, Row2 (&w0)[T],
+                                         Row2 (&w1)[T], float*& out, size_t pitch, double& acc, RowRange& rng) {
   constexpr int ST = kStageFloats<G>;
   const bool lane0 = (threadIdx.x & 31) == 0;
 #if UC_RING_TEST_AHEAD
-  bool ready = false;  // row u's phase already observed complete by the previous step's test
+  bool ready = false;
 #endif
 #pragma unroll
   for (int u = 0; u < kGroup; ++u) {
-    float L[T], R[T];
-    t_neighbours<T, 0, HOIST>(w1, L, R);
+    pair_t lr[T];
+    t_neighbours2<T, 0, HOIST>(w1, lr);
 #if UC_RING_TEST_AHEAD
     mbar_wait_unless(full + u, ph, ready);
 #else
     mbar_wait(full + u, ph);
 #endif
-    const float4 nv = *reinterpret_cast<const float4*>(ringp + u * ST);
+    const float4 n = *reinterpret_cast<const float4*>(ringp + u * ST);
+    if (SC) range_add(rng, n);
+    const Row2 nv = ring_row2<DIRI>(n);
     __syncwarp();
     mbar_arrive_if(empty + u, lane0);
 #if UC_RING_TEST_AHEAD
-    if (u + 1 < kGroup) ready = mbar_test(full + u + 1, ph);  // answered while this row computes
+    if (u + 1 < kGroup) ready = mbar_test(full + u + 1, ph);
 #endif
-    t_neighbours<T, HOIST, T>(w1, L, R);
-    t_levels<T, NL, DIRI, true>(nv, g, nx4, a, b, i0 + u, w0, w1, L, R, out, pitch, acc);
+    t_neighbours2<T, HOIST, T>(w1, lr);
+    t_levels2<T, NL, DIRI, true, SC>(nv, g, nx4, a, b, i0 + u, w0, w1, lr, out, pitch, acc);
   }
 }
 
-template <int T, int NL, bool DIRI, int G>
-__device__ __forceinline__ void march_t(const JacobiParams& p, const float* src, float* dst, int s,
+// The march of one block over A_{k+T} rows a..b.  gi0: ring rows this block has already used in
+// this launch (a re-run continues the ring's stage and phase sequence).  SC: the scaled march;
+// returns true when this warp saw an A_k value outside its range (consumers only).
+template <int T, int NL, bool DIRI, int G, bool SC>
+__device__ __forceinline__ bool march_t(const JacobiParams& p, const float* src, float* dst, int s,
                                         const GhostLayout& g, int a, int b, double& acc, float* ring,
-                                        uint64_t* full, uint64_t* empty, bool proxy_fence) {
+                                        uint64_t* full, uint64_t* empty, bool proxy_fence, int gi0) {
   const int nc = p.consumers, NS = p.stages;
   constexpr int PAD = Ghost<G>::kPadG;
 #if UC_MARCH_GROUPED
@@ -417,10 +577,10 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
       const uint64_t pol = policy_evict_normal();
 #endif
       if (proxy_fence) fence_proxy_async_global();
-      int st = 0;
-      unsigned ph = 0;
+      int st = gi0 % NS;
+      unsigned ph = (unsigned)(gi0 / NS) & 1u;
       for (int i = 0; i < rows; ++i) {
-        if (i >= NS) mbar_wait(empty + st, ph ^ 1u);
+        if (gi0 + i >= NS) mbar_wait(empty + st, ph ^ 1u);
         mbar_arrive_expect_tx(full + st, bytes);
 #ifdef UC_PROTO_L2_ROWS  // A/B measurement only (scripts/proto): cycle over a few L2-resident rows
         bulk_g2s(ring + (size_t)st * ST + off, src + (size_t)(a - T + i % UC_PROTO_L2_ROWS) * pitch + left, bytes,
@@ -434,29 +594,29 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
         }
       }
     }
-    return;
+    return false;
   }
   const int nx4 = p.nx4;
-  float4 w0[T], w1[T];  // level j: rows r-j-1 (w0) and r-j (w1) before row r arrives
+  Row2 w0[T], w1[T];  // level j: rows r-j-1 (w0) and r-j (w1) before row r arrives
 #pragma unroll
-  for (int j = 0; j < T; ++j) w0[j] = w1[j] = make_float4(0.f, 0.f, 0.f, 0.f);
-  RingCursor cur{0, 0u};
+  for (int j = 0; j < T; ++j) w0[j] = w1[j] = Row2{0ull, 0ull};
+  RowRange rng{0.f, ~0u};
+  RingCursor cur{gi0 % NS, (unsigned)(gi0 / NS) & 1u};
+  constexpr int H = kHoistLevels<T, G>;
   float* out = dst + (size_t)a * pitch + 4 * (size_t)g.x4;  // the A_{k+T} row a comes out at i = 2T
   // the first 2T rows only fill the levels (rows >= 2T + 1 since a <= b)
 #pragma unroll
   for (int i = 0; i < 2 * T; ++i)
-    t_step<T, NL, DIRI, false, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
-                                                      pitch, acc);
+    t_step2<T, NL, DIRI, false, H, SC>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc, rng);
 #if UC_MARCH_GROUPED
   int i = 2 * T;
   // single rows up to the next group boundary (ring stage 0 mod kGroup)
   for (; i < rows && cur.st % kGroup != 0; ++i)
-    t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
-                                                     pitch, acc);
+    t_step2<T, NL, DIRI, true, H, SC>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc, rng);
   const float* ringl = ring + g.ring_off;
   for (; i + kGroup <= rows; i += kGroup) {
-    t_group<T, NL, DIRI, G, kHoistLevels<T, G>>(ringl + cur.st * ST, full + cur.st, empty + cur.st, cur.ph, g, nx4,
-                                                a, b, i, w0, w1, out, pitch, acc);
+    t_group2<T, NL, DIRI, G, H, SC>(ringl + cur.st * ST, full + cur.st, empty + cur.st, cur.ph, g, nx4, a, b, i, w0,
+                                    w1, out, pitch, acc, rng);
     cur.st += kGroup;
     if (cur.st == NS) {
       cur.st = 0;
@@ -464,14 +624,14 @@ __device__ __forceinline__ void march_t(const JacobiParams& p, const float* src,
     }
   }
   for (; i < rows; ++i)
-    t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
-                                                     pitch, acc);
+    t_step2<T, NL, DIRI, true, H, SC>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc, rng);
 #else
 #pragma unroll(kTUnroll)
   for (int i = 2 * T; i < rows; ++i)
-    t_step<T, NL, DIRI, true, kHoistLevels<T, G>>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out,
-                                                     pitch, acc);
+    t_step2<T, NL, DIRI, true, H, SC>(ring, full, empty, ST, NS, g, nx4, a, b, i, cur, w0, w1, out, pitch, acc, rng);
 #endif
+  // a warp whose lanes are all outside the grid (the tail of the last strip) computes nothing kept
+  return SC && g.in_grid && !range_ok<T>(rng);
 }
 
 // Boundary rounds 2..T after the march, out of line: the march's register allocation then does not
@@ -536,8 +696,17 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
     // in profiles/r2_trace_blocks.txt).  The producer warp's path is the same in both instances.
     const int wx0 = xs4 + warp_id_uniform() * Ghost<G>::kOwn - G;  // float4 column of lane 0
     const bool diri = (wx0 <= 0 && 0 < wx0 + 32) || (wx0 <= p.nx4 - 1 && p.nx4 - 1 < wx0 + 32);
-    if (diri) march_t<T, NL, true, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
-    else march_t<T, NL, false, G>(p, src, dst, s, g, a, b, acc, ring, full, empty, top_blk || bot_blk);
+    const bool pf = top_blk || bot_blk;
+    constexpr bool kScaled = UC_SCALED_MARCH && NL == 0;
+    bool bad = false;
+    if (diri) march_t<T, NL, true, G, false>(p, src, dst, s, g, a, b, acc, ring, full, empty, pf, 0);
+    else bad = march_t<T, NL, false, G, kScaled>(p, src, dst, s, g, a, b, acc, ring, full, empty, pf, 0);
+    if (kScaled && __syncthreads_or(bad)) {  // a value outside the scaled range: redo unscaled
+      if (threadIdx.x == 0) atomicAdd(p.launch_hist + 15, 1ull);  // uc_jacobi_launch_counts()[15]
+      const int gi = b - a + 1 + 2 * T;
+      if (diri) march_t<T, NL, true, G, false>(p, src, dst, s, g, a, b, acc, ring, full, empty, false, gi);
+      else march_t<T, NL, false, G, false>(p, src, dst, s, g, a, b, acc, ring, full, empty, false, gi);
+    }
   }
   UC_TRACE_AT(2);
   if ((rtop || rbot) && (int)threadIdx.x < p.consumers) {

@@ -64,7 +64,8 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
             pm = MODES[mode] | (U.UC_PLAN_DEEP_HALO if host_path and host_path[0] and mode == "host" else 0)
             want = expected_counts(U, info, pm, ny // P, iters, norm_every, stepwise, chunks_of_run)
             if want is not None:  # the launches that really ran are the plan's (no silent demotion)
-                assert counts == want, (f"rank {rank}: launches by iterations per launch {counts[:9]} != "
+                # (slot 15 counts blocks whose scaled march re-ran unscaled, not launches)
+                assert counts[:15] == want[:15], (f"rank {rank}: launches by iterations per launch {counts[:9]} != "
                                         f"plan {want[:9]} ({info})")
             return slab0, final, norms, info, counts
         finally:

@@ -70,7 +70,7 @@ def test_weak_scaling_8x16384sq_sampled_rows(variant, k, ne):
     if variant == 5:
         for r in range(P):
             c = res[r][4]
-            assert (c[6], sum(c)) == ((2, 2) if k == 12 else (0, 1)), c
+            assert (c[6], sum(c[:15])) == ((2, 2) if k == 12 else (0, 1)), c
     for r in range(P):
         top, bot, mid, _, _ = res[r]
         g0 = r * n  # global computed row of slab row 1

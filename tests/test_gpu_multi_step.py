@@ -239,7 +239,7 @@ def test_t6_config1():
     before it)."""
     res = _check(4096, 4096, 2, "ring", "device", 1000, norm_every=100, **_v5(6))
     for c in res["counts_all"]:
-        assert c[6] == 165 and c[5] == 2 and sum(c) == 167, c
+        assert c[6] == 165 and c[5] == 2 and sum(c[:15]) == 167, c
 
 
 @pytest.mark.parametrize("T", DEEP)
@@ -327,3 +327,65 @@ def test_t6_injected_flag_latency(monkeypatch, P, topology):
     monkeypatch.setenv("UC_INJECT_PUT_DELAY_NS", "20000")
     res = _check(1028, 32 * P, P, topology, "device", 24, norm_every=8)
     assert all(c[8] == 3 for c in res["counts_all"])
+
+
+# --------------------------------------------------------------------------- the scaled march
+# Norm-free T-level launches drop the 0.25 products of levels 1..T-1: exact only
+# while every nonzero |A_k| a warp reads lies in [2^(-103+2T), 2^110).  Outside that range the
+# block re-runs its march unscaled; the device counts those blocks (launch_counts()[15]).  Each
+# case below is bit-exact against the oracle AND checks which path ran.
+def _scaled_case(nx, ny, P, T, iters, init, topology="ring"):
+    _, want, _ = _oracle(nx, ny, topology, iters, 0, init=init)
+    res = solve_gpu(nx, ny, P, topology, "device", iters, 0, init=init, **_v5(T))
+    assert_slabs_equal_global(res["final"], want, P, topology)
+    return [c[15] for c in res["counts_all"]]
+
+
+@pytest.mark.parametrize("T", [6, 8])
+def test_scaled_march_runs_on_ordinary_fields(T):
+    """The generator's field (values in [0, 1) on a 2^-24 grid): no block leaves the scaled march."""
+    from inputs import gen
+    g = gen.global_field(2052, 96, "ring")
+    assert _scaled_case(2052, 96, 2, T, 3 * T, g) == [0, 0]
+
+
+@pytest.mark.parametrize("T", [6, 8])
+@pytest.mark.parametrize("scale_log2", [-100, -60, 100, 112])
+def test_scaled_march_falls_back_outside_its_range(T, scale_log2):
+    """One launch of the generator's field scaled by 2^s (nonzero |values| in [2^(s-24), 2^s)).
+    2^-100: tiny but normal, the unscaled iteration's values can reach the subnormal range within
+    T levels; 2^112: scaled sums could overflow -- every interior block re-runs unscaled.  2^-60
+    and 2^100 are inside [2^(-103+2T), 2^110) for T <= 8: no re-run."""
+    from inputs import gen
+    g = gen.global_field(2052, 96, "ring")
+    g = (g.astype(np.float64) * 2.0 ** scale_log2).astype(np.float32)
+    reruns = _scaled_case(2052, 96, 2, T, T, g)
+    if -103 + 2 * T <= scale_log2 - 24 and scale_log2 < 110:
+        assert reruns == [0, 0], reruns
+    else:
+        assert all(r > 0 for r in reruns), reruns
+
+
+@pytest.mark.parametrize("T", [6, 8])
+def test_scaled_march_spike_into_the_subnormals(T):
+    """A single 1.0 in an interior column of a zero field, 12 launches: the front of the diamond
+    decays by 4 per iteration into the subnormal range (2^-2k at distance k), so later launches
+    meet values below 2^(-103+2T) in the blocks around the spike and re-run them unscaled, while
+    far blocks stay scaled.  Bit-exact (no FTZ, no scaling error) either way."""
+    nx, ny = 1028, 128
+    a = np.zeros((ny + 2, nx), np.float32)
+    a[64, 520] = 1.0
+    reruns = _scaled_case(nx, ny, 1, T, 12 * T, a)
+    assert reruns[0] > 0
+
+
+@pytest.mark.parametrize("T", [8])
+def test_scaled_march_inf_and_huge(T):
+    """+inf and 2^126 values in one interior point: inf is out of the scaled range (re-run);
+    the unscaled iteration spreads inf and large finite values exactly as the oracle does."""
+    from inputs import gen
+    g = gen.global_field(2052, 64, "ring")
+    g[20, 700] = np.float32(np.inf)
+    g[40, 1500] = np.float32(2.0 ** 126)
+    reruns = _scaled_case(2052, 64, 1, T, 3 * T, g)
+    assert reruns[0] > 0

@@ -62,11 +62,11 @@ def test_multiprocess_ipc_deep(tmp_path, P, topology):
     res = _run(tmp_path, P, 1028, 16 * P, 24, 8, topology, "device")
     for x in res:
         c = list(x["counts"])
-        assert c[8] == 3 and sum(c) == 3, c
+        assert c[8] == 3 and sum(c[:15]) == 3, c
     res = _run(tmp_path, P, 1028, 16 * P, 24, 6, topology, "device")
     for x in res:
         c = list(x["counts"])
-        assert c[6] == 4 and sum(c) == 4, c
+        assert c[6] == 4 and sum(c[:15]) == 4, c
 
 
 # ---- one GPU per rank (NCCL allows one rank per GPU): run where the box has >= 2 GPUs
