@@ -66,6 +66,8 @@ def parse():
                     help="TEST ONLY: put every rank on cuda:0 (exercises the multi-process path on a 1-GPU box; "
                          "ranks time-slice the GPU, so the numbers are not a benchmark)")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
+    ap.add_argument("--balance", action="store_true",
+                    help="balanced row chunks (uc_jacobi_set_balance 1; default: static equal chunks)")
     ap.add_argument("--halo-only", action="store_true", help="skip e2e / cpu_baseline, keep the halo leg")
     ap.add_argument("--cpu-sample-iters", type=int, default=12)
     ap.add_argument("--variant", type=int, default=-1,
@@ -240,6 +242,8 @@ def run_ours(a):
     host_path = tuple(int(x) for x in a.host_path.split(","))
     if a.mode == "host":
         J.set_host_path(*host_path)
+    if a.balance:
+        J.set_balance(True)
     n = J.n
     launch_info = J.launch_info()
     use_graph = not a.no_graph
@@ -332,12 +336,15 @@ def run_ours(a):
     achieved = alg_bytes / (k_plain / 1e3) / 1e9
     sms = torch.cuda.get_device_properties(local).multi_processor_count
     alu_peak = sms * 128 * sm_max_mhz() * 1e6 / 1e12
-    # FP32 work: 4 operations per point-iteration (3 FADD + 1 FMUL, never fused), T per launch,
-    # ghost lanes compute too (x 32 / (32 - 2G) for variant 5)
-    ops = 4.0 * pts_rank * per_launch * (32.0 / (32 - 2 * ghosts) if v == 5 else 1.0)
+    # FP32 work: the method does 4 operations per point-iteration (3 FADD + 1 FMUL, never fused).
+    # The T-level kernel's norm-free launches run the scaled march: 3 adds per level,
+    # the 4^-T product once on the last level, one exact permutation add (x + -0) as a row leaves
+    # the ring -- 3T + 2 operations per point and launch; ghost lanes compute too (x 32 / (32 - 2G))
+    alg_ops = 4.0 * pts_rank * per_launch
+    ops = ((3.0 * per_launch + 2.0) * pts_rank * 32.0 / (32 - 2 * ghosts)) if v == 5 else alg_ops
     alu = ops / (k_plain / 1e3) / 1e12
     # the two roofs as GLUPS ceilings at this depth: HBM moves 8/T B per point-iteration; the
-    # FP32 pipe does 4 (x ghost share) operations per point-iteration.  bound = the tighter one.
+    # FP32 pipe does (3T + 2)/T (x ghost share) operations per point-iteration.  bound = the tighter one.
     hbm_glups = peak / (8.0 / per_launch)
     alu_glups = alu_peak * 1e3 / (ops / (pts_rank * per_launch))
     tighter = "hbm" if hbm_glups <= alu_glups else "alu"
@@ -356,7 +363,7 @@ def run_ours(a):
         roof.update({"achieved": round(alu, 3), "peak": round(alu_peak, 2), "unit": "TFLOP/s",
                      "frac": round(alu / alu_peak, 4)})
     roof["alu"] = {"bound": "alu", "achieved": round(alu, 3), "peak": round(alu_peak, 2), "unit": "TFLOP/s",
-                   "frac": round(alu / alu_peak, 4), "flops_per_launch": ops,
+                   "frac": round(alu / alu_peak, 4), "flops_per_launch": ops, "alg_flops_per_launch": alg_ops,
                    "peak_source": f"{sms} SMs x 128 FP32 lanes x {sm_max_mhz():.0f} MHz (derived, DESIGN.md §5)"}
     roof["hbm"] = {"achieved": round(achieved, 1), "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4)}
 
@@ -385,6 +392,8 @@ def run_ours(a):
             J2.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages, a.tile_rows)
         if a.mode == "host":
             J2.set_host_path(*host_path)
+        if a.balance:
+            J2.set_balance(True)
         stream2 = torch.cuda.Stream()
         coord2 = U.Coord(comm, mode, stream2.cuda_stream)
         h_in = torch.empty(slab_elems, dtype=torch.float32, pin_memory=True)
@@ -460,7 +469,7 @@ def run_ours(a):
                                      else None),
                        "parallelism": f"y-slab x{world}", "l2": "inputs > L2 (2 slabs x "
                        f"{(n + 2) * nx * 4 / 2**20:.0f} MiB per GPU vs 126 MB L2), no flush",
-                       "launch": launch_info},
+                       "launch": launch_info, "balanced_chunks": bool(v == 5 and a.mode == "device" and a.balance)},
             "roofline": roof, "cpu_baseline": cpu, "cpu_parallel": cpu_par, "e2e": e2e, "clocks": clk, "gpu_launches": launches,
             "gpu_launches_by_depth": {str(d): c for d, c in enumerate(ran) if c},
             "scaled_march_reruns": reruns,

@@ -83,6 +83,10 @@ _SIGS = {
     "uc_jacobi_num_norms": (i32, [vp, i32, i32]),
     "uc_jacobi_launch_counts": (i32, [vp, P(u64), i32]),
     "uc_jacobi_set_host_path": (i32, [vp, i32, i32]),
+    "uc_jacobi_set_balance": (i32, [vp, i32]),
+    "uc_jacobi_balance_rates": (i32, [vp, vp, dp, i32]),
+    "uc_jacobi_balance_table": (i32, [vp, P(i32), i32, P(i32)]),
+    "uc_balance_plan": (i32, [i32, i32, i32, i32, i32, dp, P(i32)]),
     "uc_jacobi_solve": (i32, [vp, vp, i32, i32, C.c_double, P(i64), dp]),
     "uc_coord_set_p2p_path": (i32, [vp, i32, i32]),
     "uc_jacobi_launch_plan": (i32, [i32, i32, i32, i32, i32, i32, P(i32), i32]),

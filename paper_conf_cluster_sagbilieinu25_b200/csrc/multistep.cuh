@@ -383,7 +383,7 @@ __device__ __forceinline__ float4 t_fetch(const float* ring, uint64_t* full, uin
 #define UC_HOIST_62 3  // levels hoisted at <6, 2> (A/B: 0 / 2 / 3 / 4 -> 3509 / 3546 / 3568 / 3530 GLUPS)
 #endif
 #ifndef UC_HOIST_82
-#define UC_HOIST_82 2  // levels hoisted at <8, 2> (A/B, march alone: 0/2/3/4/8 -> 0.492/0.487/0.489/0.488/0.536 ms: hoisting all spills)
+#define UC_HOIST_82 8  // levels hoisted at <8, 2> (A/B in the pair frame + scaled march, profiles/r2_pq_scaled_ab.txt: 0/2/4/8 -> 0.446/0.443/0.443/0.439 ms)
 #endif
 #ifndef UC_HOIST_72
 #define UC_HOIST_72 7  // levels hoisted at <7, 2> (A/B)
@@ -653,19 +653,30 @@ __device__ __noinline__ double t_rounds_after(const JacobiParams& p, const float
 
 template <int T, int NL, int G>
 __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int par, float* ring, uint64_t* full,
-                                         uint64_t* empty) {
+                                         uint64_t* empty, unsigned long long t_entry = 0) {
   constexpr int PT = T > 1 ? T - 1 : 1;
   const float* src = p.slab[par];
   float* dst = p.slab[par ^ 1];
-  const int s = blockIdx.x % p.strips;
-  // part 0: every row chunk; part 1 (host overlap): the first and last chunk only (grid 2 x strips);
-  // part 2: the others (chunks 1..chunks-2)
-  const int q = p.part == 0 ? blockIdx.x / p.strips
-                : p.part == 1 ? (blockIdx.x < p.strips ? 0 : p.chunks - 1)
-                              : blockIdx.x / p.strips + 1;
+  int s, q, lo, hi;
+  if (NL == 0 && p.bal_tab != nullptr) {
+    // balanced launch: this block's (strip, chunk, rows) from the table uc_jacobi_run maintains
+    // (any partition of every strip's rows into its chunks in order is exact; norm launches keep
+    // the static chunking, so the block partials -- and the norm -- do not depend on timing)
+    const int4 w = p.bal_tab[blockIdx.x];
+    s = w.x;
+    q = w.y;
+    lo = w.z;
+    hi = w.w;
+  } else {
+    s = blockIdx.x % p.strips;
+    // part 0: every row chunk; part 1 (host overlap): the first and last chunk only (grid 2 x strips);
+    // part 2: the others (chunks 1..chunks-2)
+    q = p.part == 0 ? blockIdx.x / p.strips
+        : p.part == 1 ? (blockIdx.x < p.strips ? 0 : p.chunks - 1)
+                      : blockIdx.x / p.strips + 1;
+    chunk_rows(p, q, lo, hi);
+  }
   const GhostLayout g = ghost_layout<G>(p, s);
-  int lo, hi;
-  chunk_rows(p, q, lo, hi);
   const bool top_blk = q == 0, bot_blk = q == p.chunks - 1;
   // deep-halo host mode: a side with a neighbour holds T halo rows of A_k (the host exchanged T
   // rows), so the march covers the edge rows too (it streams rows 1-T..0 / n+1..n+T) and that
@@ -708,6 +719,12 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
       else march_t<T, NL, false, G, false>(p, src, dst, s, g, a, b, acc, ring, full, empty, false, gi);
     }
   }
+  if (NL == 0 && p.bal_ns != nullptr && T == p.bal_T) {
+    // the block's march time (kernel entry to the end of its march: round 1 included, the later
+    // rounds not -- the first/last chunks' allowance for them is the static chunk_shrink)
+    __syncthreads();
+    if (threadIdx.x == 0) p.bal_ns[blockIdx.x] = globaltimer() - t_entry;
+  }
   UC_TRACE_AT(2);
   if ((rtop || rbot) && (int)threadIdx.x < p.consumers) {
 #if UC_ROUNDS_NOINLINE
@@ -731,6 +748,74 @@ __device__ __forceinline__ double t_body_nl(const JacobiParams& p, uint64_t k, i
     if (nl != NL) return t_body_nl<T, NL + 1, G>(p, k, par, ring, full, empty, nl);
   }
   return t_body<T, NL, G>(p, k, par, ring, full, empty);
+}
+
+// Balanced chunks: the last block of a timed launch folds every block's march time
+// into its rate (rows per ns, smoothed 1:1 with the previous value) and re-cuts each strip's rows
+// among its chunks in proportion to the rates of the blocks serving them: sizes in effective rows
+// (E = n + 2 shrink, the first/last chunk carrying the static allowance for their boundary rounds),
+// water-filled above per-chunk minimums (first/last levels + 1 rows, others levels, +1 of slack
+// for the floor of the cumulative cuts), so a non-edge chunk never reaches a halo row.  Thread s
+// cuts strip s; scratch: the block's ring (free after its march).
+static __device__ __noinline__ void bal_resize(const JacobiParams& p, unsigned char* scratch, size_t scratch_bytes) {
+  const int S = p.strips, Q = p.chunks, NG = S * Q;
+  if ((size_t)NG * (sizeof(double) + 1) > scratch_bytes) return;  // keep the cuts (tiny rings only)
+  double* rt = reinterpret_cast<double*>(scratch);
+  unsigned char* pin = scratch + sizeof(double) * NG;
+  for (int e = threadIdx.x; e < NG; e += blockDim.x) {
+    const int b = p.bal_inv[e];
+    const int4 w = p.bal_tab[b];
+    const unsigned long long ns = p.bal_ns[b];
+    float r = p.bal_rate[b];
+    const int rows = w.w - w.z + 1;
+    if (ns > 0 && rows > 0) {
+      const float smp = (float)rows / (float)ns;
+      r = r > 0.f ? 0.5f * (r + smp) : smp;
+      p.bal_rate[b] = r;
+    }
+    rt[e] = r;
+    pin[e] = 0;
+  }
+  __syncthreads();
+  const long long E = (long long)p.n + 2LL * p.chunk_shrink;
+  for (int s = threadIdx.x; s < S; s += blockDim.x) {
+    double* r = rt + (size_t)s * Q;
+    unsigned char* pn = pin + (size_t)s * Q;
+    bool all = true;
+    double msum = 0.0;
+    for (int q = 0; q < Q; ++q) {
+      all &= r[q] > 0.0;
+      msum += Q == 1 ? (double)E : (q == 0 || q == Q - 1) ? (double)(p.chunk_shrink + p.bal_levels + 2)
+                                                            : (double)(p.bal_levels + 1);
+    }
+    if (!all || msum > (double)E) continue;  // no rates yet / no room: keep this strip's cuts
+    const auto mn = [&](int q) {
+      return Q == 1 ? (double)E : (q == 0 || q == Q - 1) ? (double)(p.chunk_shrink + p.bal_levels + 2)
+                                                         : (double)(p.bal_levels + 1);
+    };
+    double rest = 0.0, rs = 0.0;
+    for (bool again = true; again;) {
+      again = false;
+      rest = (double)E;
+      rs = 0.0;
+      for (int q = 0; q < Q; ++q) {
+        if (pn[q]) rest -= mn(q);
+        else rs += r[q];
+      }
+      for (int q = 0; q < Q; ++q)
+        if (!pn[q] && rest * r[q] / rs < mn(q)) pn[q] = 1, again = true;
+    }
+    double cum = 0.0;
+    long long prev = 0;
+    for (int q = 0; q < Q; ++q) {
+      cum += pn[q] ? mn(q) : rest * r[q] / rs;
+      const long long B = q == Q - 1 ? E : (long long)floor(cum + 1e-6);
+      const int lo = 1 + (int)max(0LL, min(prev - p.chunk_shrink, (long long)p.n));
+      const int hi = (int)max(0LL, min(B - p.chunk_shrink, (long long)p.n));
+      p.bal_tab[p.bal_inv[s * Q + q]] = make_int4(s, q, lo, hi);
+      prev = B;
+    }
+  }
 }
 
 // T iterations per launch with G ghost lanes per warp side (T <= 4G).  Device mode: n >= 2T, at
@@ -757,6 +842,7 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
     fence_mbar_init();
   }
   __syncthreads();
+  const unsigned long long t_entry = globaltimer();
   const uint64_t k = p.k_dev[0];
   const int par = (int)((k + p.k_dev[2]) & 1);
   int nl = 0;  // level (1..T) whose iteration k+nl-1 is a norm iteration
@@ -770,7 +856,7 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
   // check and every ring wait a reconvergence region)
   nl = __shfl_sync(kFull, nl, 0);
   double acc = 0.0;
-  if (nl == 0) t_body<T, 0, G>(p, k, par, ring, full, empty);
+  if (nl == 0) t_body<T, 0, G>(p, k, par, ring, full, empty, t_entry);
   else acc = t_body_nl<T, 1, G>(p, k, par, ring, full, empty, nl);
   if (nl > 0) {
     const double t = block_sum(acc, smem);
@@ -787,6 +873,10 @@ __global__ void __launch_bounds__(G == 1 ? kMaxBlock + 32 : UC_T8_MAXTHREADS, G 
   if (s_last) {
     __threadfence();
     finish_iteration(p, nl > 0, smem, T);
+    if (nl == 0 && p.bal_tab != nullptr && T == p.bal_T) {
+      __syncthreads();
+      bal_resize(p, reinterpret_cast<unsigned char*>(ring), (size_t)NS * kStageFloats<G> * sizeof(float));
+    }
   }
   UC_TRACE_AT(15);
 }

@@ -7,6 +7,7 @@
 namespace uc {
 
 #if UC_TRACE
+int set_trace_g2c(unsigned long long* buf);
 static unsigned long long* g_trace = nullptr;
 }  // namespace uc
 extern "C" unsigned long long* uc_debug_trace_buffer() { return uc::g_trace; }
@@ -19,6 +20,7 @@ int launch_jacobi_t_g2b(const JacobiParams& p, int grid, int block, int T, size_
     UC_CUDA(cudaMallocManaged(&g_trace, sizeof(unsigned long long) * 16 * 4096));
     memset(g_trace, 0, sizeof(unsigned long long) * 16 * 4096);
     UC_CUDA(cudaMemcpyToSymbol(uc_trace_ptr, &g_trace, sizeof g_trace));
+    if (int e = set_trace_g2c(g_trace)) return e;
   }
 #endif
   switch (T) {

@@ -4,6 +4,14 @@
 
 namespace uc {
 
+#if UC_TRACE
+// every translation unit has its own copy of the trace pointer (multistep.cuh): set this one too
+int set_trace_g2c(unsigned long long* buf) {
+  UC_CUDA(cudaMemcpyToSymbol(uc_trace_ptr, &buf, sizeof buf));
+  return UC_OK;
+}
+#endif
+
 int launch_jacobi_t_g2c(const JacobiParams& p, int grid, int block, size_t smem, cudaStream_t s) {
   jacobi_t_kernel<8, 2><<<grid, block, smem, s>>>(p);
   UC_CUDA(cudaGetLastError());

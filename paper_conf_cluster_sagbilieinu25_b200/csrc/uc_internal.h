@@ -75,6 +75,16 @@ struct JacobiParams {
   int partial_base;                    // index of this launch's first block partial
   unsigned put_delay_ns;               // test/measurement knob (UC_INJECT_PUT_DELAY_NS): each boundary
                                        // round's flag is released this much later (NVLink-like latency)
+  // variant 5, device mode, norm-free launches: the balanced work table (nullptr: the static
+  // chunking).  bal_tab[b] = {strip, chunk, first row, last row} of block b.  Launches of depth
+  // bal_T time each block's march; their last block folds the times into the rates and re-cuts
+  // every strip's rows in proportion to its blocks' rates
+  int4* bal_tab;
+  const int* bal_inv;                  // [strips * chunks]: block serving (strip s, chunk q) at s * chunks + q
+  unsigned long long* bal_ns;          // [grid]: block b's march time in the last launch of depth bal_T
+  float* bal_rate;                     // [grid]: block b's smoothed rate, rows per ns
+  int bal_T;
+  int bal_levels;                      // the solver's T (minimum chunk sizes)
   int gpu_scope;                       // 1: top and bottom live on this GPU (same process): halo
                                        // flags at .gpu scope instead of .sys
   double* partials;                    // local [grid] per-block partial sums
@@ -307,4 +317,29 @@ struct uc_jacobi {
   int block = 0, blocks_per_sm = 0, grid = 0, chunks = 0;
   int partials_cap = 0;
   GraphCache graphs;
+  // balanced work table (variant 5, device mode, norm-free launches): blocks are
+  // placed on SMs the same way every launch and SMs differ in speed (up to ~1.3x, measured); the
+  // table re-cuts the strips' rows in proportion to measured per-block rates.  Off by default:
+  // it equalises the blocks' finish times, but the fast SMs slow down when given more rows
+  // (the rates are shares of a common limit), so the launch gains ~2 % and the step nothing
+  int balance = 0;                         // uc_jacobi_set_balance
+  int bal_ok = 0;                          // the device table holds a valid partition
+  int bal_cap = 0;                         // capacity of the arrays below (blocks)
+  int4* bal_tab = nullptr;                 // device [cap]: {strip, chunk, first row, last row}
+  int* bal_inv = nullptr;                  // device [cap]: (strip, chunk) -> block
+  unsigned long long* bal_ns = nullptr;    // device [cap]: march ns of the last timed launch
+  float* bal_rate = nullptr;               // device [cap]: smoothed rows per ns per block
+  int4* bal_tab_h = nullptr;               // pinned staging of a table upload
+  int* bal_inv_h = nullptr;                // pinned staging of an inverse upload
+  float* bal_rate_h = nullptr;             // pinned readback of bal_rate
+  cudaEvent_t bal_ev = nullptr;            // after the readback
+  int bal_pending = 0;                     // a readback is in flight
+  int bal_T = 0;                           // the depth whose launches are timed
+  int bal_assigned = 0;                    // the host has dealt blocks to strips by measured rates
+  std::vector<int> bal_strip;              // block -> strip of the table on the device
 };
+
+// Partition each strip's n rows among its `chunks` blocks in proportion to the blocks' rates
+// (uc_balance_plan in the C-ABI; pure host logic).  Returns false when the minimum sizes do not fit.
+bool balance_plan(int strips, int chunks, int n, int shrink, int levels, const double* rate, int4* tab,
+                  const double* strip_cols = nullptr);

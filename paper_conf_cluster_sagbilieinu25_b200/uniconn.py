@@ -139,6 +139,19 @@ def launch_plan(variant: int, levels: int, mode: int, n_local: int, iters: int, 
     return list(buf[:cnt])
 
 
+def balance_plan(strips: int, chunks: int, n: int, shrink: int, levels: int, rates=None):
+    """uc_balance_plan: the balanced chunk table for per-block rates (host logic, no device);
+    returns an int array [strips * chunks, 4] of {strip, chunk, first row, last row}."""
+    import numpy as np
+    g = strips * chunks
+    tab = np.zeros((g, 4), np.int32)
+    r = None if rates is None else np.ascontiguousarray(rates, np.float64)
+    rp = None if r is None else r.ctypes.data_as(C.POINTER(C.c_double))
+    check(lib.uc_balance_plan(strips, chunks, n, shrink, levels, rp, tab.ctypes.data_as(C.POINTER(C.c_int))),
+          "uc_balance_plan")
+    return tab
+
+
 class SymMem:
     """Symmetric memory: same-size, peer-addressable on every rank."""
 
@@ -360,6 +373,27 @@ class Jacobi:
         """uc_jacobi_set_host_path (same call on every rank)."""
         check(lib.uc_jacobi_set_host_path(self.h, int(deep_halo), int(overlap)), "uc_jacobi_set_host_path")
         self.host_deep = bool(deep_halo)
+
+    def set_balance(self, enable: bool):
+        """uc_jacobi_set_balance: balanced chunks on (default) / off."""
+        check(lib.uc_jacobi_set_balance(self.h, int(enable)), "uc_jacobi_set_balance")
+
+    def balance_rates(self, coord, rates):
+        """uc_jacobi_balance_rates: install the table for these per-block rates now."""
+        import numpy as np
+        r = np.ascontiguousarray(rates, np.float64)
+        check(lib.uc_jacobi_balance_rates(coord.h, self.h, r.ctypes.data_as(C.POINTER(C.c_double)), len(r)),
+              "uc_jacobi_balance_rates")
+
+    def balance_table(self):
+        """uc_jacobi_balance_table: [grid, 4] {strip, chunk, first row, last row}, or None (static)."""
+        import numpy as np
+        g = self.launch_info()["grid"]
+        tab = np.zeros((g, 4), np.int32)
+        n = C.c_int()
+        check(lib.uc_jacobi_balance_table(self.h, tab.ctypes.data_as(C.POINTER(C.c_int)), g, C.byref(n)),
+              "uc_jacobi_balance_table")
+        return tab if n.value > 0 else None
 
     def plan(self, mode: int, iters: int, norm_every: int) -> list:
         """The launch plan uc_jacobi_run follows for this solver under a coordinator of `mode`."""

@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--nx", type=int, default=16384)
     ap.add_argument("--ny", type=int, default=16384)
     ap.add_argument("--topology", default="ring")
+    ap.add_argument("--balance", action="store_true", help="balanced chunks on (default off here)")
     a = ap.parse_args()
     env = U.Env(0, 1, 0)
     nb = U.ring_neighbours if a.topology == "ring" else U.chain_neighbours
@@ -32,10 +33,13 @@ def main():
     st = torch.cuda.Stream()
     co = U.Coord(comm, U.UC_MODE_DEVICE, st.cuda_stream)
     J = U.Jacobi(comm, a.nx, a.ny)
+    J.set_balance(a.balance)  # off: the static chunking (the estimate below assumes its rows per block)
     info = J.launch_info()
     T = info["tile_rows"]
-    for _ in range(4):
+    for _ in range(4 if not a.balance else 40):
         J.run(co, 2 * T, 0, use_graph=False)
+        if a.balance:
+            co.sync()
     co.sync()
     U.lib.uc_debug_trace_buffer.restype = C.c_void_p
     ptr = U.lib.uc_debug_trace_buffer()
@@ -80,6 +84,51 @@ def main():
     ids = np.nonzero(mid)[0][order]
     print("slowest interior blocks (block, sm, march end us):", [(int(b), int(sm[b]), round(us(t[b, 2] - t0), 1)) for b in ids[-12:]])
     print("fastest interior blocks:", [(int(b), int(sm[b]), round(us(t[b, 2] - t0), 1)) for b in ids[:12]])
+    # is a block's speed a property of its SM?  Repeat the launch and compare the per-SM mean
+    # interior march time across repetitions (and the block -> SM placement across them)
+    reps = []
+    for _ in range(3):
+        J.run(co, T, 0, use_graph=False)
+        co.sync()
+        tr = buf.astype(np.int64).copy()
+        reps.append(tr)
+    per_sm = []
+    for tr in [t] + reps:
+        d = (tr[:, 2] - tr[:, 0]).astype(np.float64)
+        m = np.full(200, np.nan)
+        for smid in np.unique(tr[:, 14]):
+            sel = (tr[:, 14] == smid) & mid
+            if sel.any():
+                m[int(smid)] = d[sel].mean()
+        per_sm.append(m)
+        same = np.mean(tr[:, 14] == t[:, 14])
+    ok = ~np.isnan(per_sm[0]) & ~np.isnan(per_sm[1])
+    cc = [np.corrcoef(per_sm[0][ok], per_sm[i][ok])[0, 1] for i in range(1, len(per_sm))]
+    print(f"block -> SM placement identical across launches: {same:.3f}; per-SM mean interior march time "
+          f"correlation launch 0 vs 1..3: {[round(c, 3) for c in cc]}")
+    allm = np.nanmean(np.array(per_sm), axis=0)
+    okm = ~np.isnan(allm)
+    ids_sm = np.nonzero(okm)[0]
+    v = allm[okm] / 1e3
+    print(f"per-SM mean interior march (us, 4 launches): min {v.min():.1f} median {np.median(v):.1f} max {v.max():.1f}; "
+          f"slowest SMs {[int(x) for x in ids_sm[np.argsort(v)[-10:]]]}, fastest {[int(x) for x in ids_sm[np.argsort(v)[:10]]]}")
+    print("per-SM mean interior march (us) by SM id:", " ".join(f"{int(i)}:{x:.0f}" for i, x in zip(ids_sm, v)))
+    # what balancing could buy: per block rate = march rows / march time (mean over the launches);
+    # (a) the launch now (slowest march end), (b) rows re-cut within each strip (blocks keep their
+    # strips), (c) fully balanced (total rows / summed rates)
+    d = np.mean([(tr[:, 2] - tr[:, 0]).astype(np.float64) for tr in [t] + reps], axis=0) / 1e3
+    rows = np.zeros(info["grid"])
+    n = J.n
+    for b in range(info["grid"]):
+        qb = b // S
+        lo = 1 + max(0, min(qb * (n + 2 * 160) // Q - 160, n)) if Q > 2 else 1 + qb * n // Q
+        hi = max(0, min((qb + 1) * (n + 2 * 160) // Q - 160, n)) if Q > 2 else (qb + 1) * n // Q
+        rows[b] = hi - lo + 1
+    rate = rows / d
+    strip_t = [rows[q * S + s_] .sum() if False else None for s_ in range(S) for q in range(1)]
+    per_strip = [rows[np.arange(s_, info["grid"], S)].sum() / rate[np.arange(s_, info["grid"], S)].sum() for s_ in range(S)]
+    print(f"balancing estimate (march us): now max {d.max():.1f} (median {np.median(d):.1f}); rows re-cut within "
+          f"strips: {max(per_strip):.1f}; fully balanced: {rows.sum() / rate.sum():.1f}")
     J.destroy()
     co.destroy()
     comm.destroy()

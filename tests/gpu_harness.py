@@ -18,7 +18,7 @@ def neighbours(U, topology):
 def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0, seed=gen.DEFAULT_SEED,
               zero_init=False, init=None, use_graph=True, stepwise=False, block_x=0, blocks_per_sm=0,
               variant=-1, stages=0, tile_rows=0,
-              chunks_of_run=None, host_path=None):
+              chunks_of_run=None, host_path=None, balance=None, balance_rates=None):
     """Returns dict(init=[slab0 per rank], final=[slab per rank], norms=np.array (rank 0),
     norms_all=[per rank], launch=launch_info of rank 0)."""
     import torch
@@ -38,6 +38,10 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
                 J.set_launch(variant, block_x, blocks_per_sm, stages, tile_rows)
             if host_path is not None:
                 J.set_host_path(*host_path)
+            if balance is not None or balance_rates is not None:
+                J.set_balance(True if balance is None else balance)
+            if balance_rates is not None:  # a callable: (rank, grid) -> per-block rates
+                J.balance_rates(coord, balance_rates(rank, J.launch_info()["grid"]))
             slab0 = J.copy_out()
             if init is not None:
                 J.copy_in(gen.rank_slab(init, rank, P))
@@ -67,7 +71,7 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
                 # (slot 15 counts blocks whose scaled march re-ran unscaled, not launches)
                 assert counts[:15] == want[:15], (f"rank {rank}: launches by iterations per launch {counts[:9]} != "
                                         f"plan {want[:9]} ({info})")
-            return slab0, final, norms, info, counts
+            return slab0, final, norms, info, counts, J.balance_table()
         finally:
             comm.barrier()
             J.destroy()
@@ -78,7 +82,7 @@ def solve_gpu(nx, ny, P, topology="ring", mode="device", iters=10, norm_every=0,
     res = run_ranks(P, body)
     return {"init": [r[0] for r in res], "final": [r[1] for r in res], "norms": res[0][2],
             "norms_all": [r[2] for r in res], "launch": res[0][3], "counts": res[0][4],
-            "counts_all": [r[4] for r in res]}
+            "counts_all": [r[4] for r in res], "balance_tables": [r[5] for r in res]}
 
 
 def expected_counts(U, info, mode, n_local, iters, norm_every, stepwise=False, chunks_of_run=None):

@@ -389,3 +389,48 @@ def test_scaled_march_inf_and_huge(T):
     g[40, 1500] = np.float32(2.0 ** 126)
     reruns = _scaled_case(2052, 64, 1, T, 3 * T, g)
     assert reruns[0] > 0
+
+
+# --------------------------------------------------------------------------- balanced chunks
+# Device-mode T-level launches without a norm round take each block's (strip, chunk, rows) from
+# a table re-partitioned from measured per-block march times.  Any valid table
+# computes the same grid; norm launches keep the static chunking, so norms are independent of it.
+def _rand_rates(seed):
+    def f(rank, grid):
+        rng = np.random.default_rng(seed + 7 * rank)
+        return rng.uniform(0.2, 5.0, grid)
+    return f
+
+
+@pytest.mark.parametrize("T", [6, 8])
+@pytest.mark.parametrize("P,topology", [(1, "ring"), (2, "ring"), (3, "dirichlet")])
+def test_balanced_table_any_partition_is_exact(T, P, topology):
+    """Wildly unequal forced rates (0.2 .. 5): blocks change strips and chunk sizes; grid bit-exact,
+    norms bit-identical to the static chunking's (norm launches do not use the table)."""
+    nx, ny, iters, ne = 2052, 1024 * P, 5 * T + 3, 2 * T
+    res = _check(nx, ny, P, topology, "device", iters, norm_every=ne, balance_rates=_rand_rates(11), **_v5(T))
+    tabs = res["balance_tables"]
+    assert all(t is not None for t in tabs)
+    info = res["launch"]
+    for t in tabs:  # the table is a partition of every strip's rows, chunks in order
+        assert sorted(map(tuple, t[:, :2].tolist())) == [(s, q) for s in range(info["strips"])
+                                                         for q in range(info["chunks"])]
+        assert not np.array_equal(t[:, 0], np.arange(len(t)) % info["strips"])  # not the static one
+    ref = solve_gpu(nx, ny, P, topology, "device", iters, ne, balance=False, **_v5(T))
+    assert ref["balance_tables"][0] is None
+    assert np.array_equal(bits(res["norms"]), bits(ref["norms"]))
+
+
+@pytest.mark.parametrize("T", [8])
+def test_balance_adapts_over_runs_and_stays_exact(T):
+    """Several runs: the table moves away from the equal split as measured rates come in (every
+    run after the first reads the previous run's block times back), and every run is bit-exact.
+    With equal rates the inner chunks of a strip differ by at most one row; SMs differ in speed
+    by far more than that, so the adapted sizes spread."""
+    nx, ny = 4100, 2048
+    res = _check(nx, ny, 1, "ring", "device", 16 * T, norm_every=0, chunks_of_run=[2 * T] * 8, balance=True,
+                 **_v5(T))
+    t = res["balance_tables"][0]
+    assert t is not None
+    inner = [r[3] - r[2] + 1 for r in t if 0 < r[1] < res["launch"]["chunks"] - 1]
+    assert max(inner) - min(inner) > 2, (min(inner), max(inner))
