@@ -38,24 +38,33 @@ def main():
           dict(P=3, mode="device", variant=5, T=6, ne=6, iters=12),
           dict(P=1, mode="device", variant=5, T=8, ne=8, iters=17), dict(P=2, mode="device", variant=5, T=8, ne=0, iters=16),
           dict(P=3, mode="device", variant=5, T=8, ne=8, iters=16)]
+    # round 2: the pair-frame march and the scaled march run in warps without a fixed column, so
+    # rows wide enough for interior warps (nx = 1028: 257 float4 columns, 2 strips); norm-free
+    # launches (scaled) and a forced balanced-chunk table
+    t6 += [dict(P=1, mode="device", variant=5, T=8, ne=0, iters=16, nx=1028, ny=64),
+           dict(P=2, mode="device", variant=5, T=8, ne=0, iters=24, nx=1028, ny=64, balance=True),
+           dict(P=3, mode="device", variant=5, T=6, ne=0, iters=12, nx=1028, ny=64)]
     if os.environ.get("UC_SANITIZE_T6_ONLY"):
         cases = t6
     else:
         cases += t6
     if len(sys.argv) > 1:
         cases = cases[: int(sys.argv[1])]
-    nx, ny = 132, 24
     for c in cases:
         P = c["P"]
+        nx, ny = c.get("nx", 132), c.get("ny", 24)
         iters = c.get("iters", 9)
         ne = c.get("ne", 2)
+        extra = {}
+        if c.get("balance"):
+            extra["balance_rates"] = lambda rank, grid: [1.0 + 0.5 * ((b * 7 + rank) % 5) for b in range(grid)]
         res = solve_gpu(nx, ny * P, P, "ring", c["mode"], iters, ne if c["mode"] != "partial" or P == 1 else 0,
-                        variant=c["variant"], tile_rows=c.get("T", 0), use_graph=False)
+                        variant=c["variant"], tile_rows=c.get("T", 0), use_graph=False, **extra)
         want, _ = oracle.jacobi_run(gen.global_field(nx, ny * P, "ring"), iters, "ring")
         assert_slabs_equal_global(res["final"], want, P, "ring")
         if c["variant"] == 5 and c.get("T", 0) in (6, 8):
             import paper_conf_cluster_sagbilieinu25_b200 as U
-            plan = U.launch_plan(5, c["T"], 1, ny, iters, ne)
+            plan = U.launch_plan(5, c["T"], 1, ny, iters, ne)  # ny = rows per rank
             assert plan[0] == c["T"], plan
         print("ok", c, flush=True)
     print("SANITIZE_RUN_DONE")
