@@ -66,6 +66,8 @@ def parse():
                     help="TEST ONLY: put every rank on cuda:0 (exercises the multi-process path on a 1-GPU box; "
                          "ranks time-slice the GPU, so the numbers are not a benchmark)")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / halo legs")
+    ap.add_argument("--e2e-streams", type=int, default=3,
+                    help="e2e leg: solvers (one stream each) whose steps are in flight at once")
     ap.add_argument("--balance", action="store_true",
                     help="balanced row chunks (uc_jacobi_set_balance 1; default: static equal chunks)")
     ap.add_argument("--halo-only", action="store_true", help="skip e2e / cpu_baseline, keep the halo leg")
@@ -386,60 +388,66 @@ def run_ours(a):
     e2e = None
     if not a.no_extras and not a.halo_only:
         slab_elems = (n + 2) * nx
-        ke = max(4, min(a.steps, 6))
-        J2 = U.Jacobi(comm, nx, ny)
-        if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages or a.tile_rows:
-            J2.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages, a.tile_rows)
-        if a.mode == "host":
-            J2.set_host_path(*host_path)
-        if a.balance:
-            J2.set_balance(True)
-        stream2 = torch.cuda.Stream()
-        coord2 = U.Coord(comm, mode, stream2.cuda_stream)
+        S = max(1, a.e2e_streams)  # solvers in flight, one stream each
+        ke = max(2 * S, min(a.steps, 3 * S))
+        solvers = [(J, coord, stream)]
+        for _ in range(S - 1):
+            Jx = U.Jacobi(comm, nx, ny)
+            if a.block_x or a.blocks_per_sm or a.variant >= 0 or a.stages or a.tile_rows:
+                Jx.set_launch(a.variant, a.block_x, a.blocks_per_sm, a.stages, a.tile_rows)
+            if a.mode == "host":
+                Jx.set_host_path(*host_path)
+            if a.balance:
+                Jx.set_balance(True)
+            sx = torch.cuda.Stream()
+            solvers.append((Jx, U.Coord(comm, mode, sx.cuda_stream), sx))
         h_in = torch.empty(slab_elems, dtype=torch.float32, pin_memory=True)
         h_in.numpy()[:] = J.copy_out(coord).ravel()
-        h_out = [torch.empty(slab_elems, dtype=torch.float32, pin_memory=True) for _ in range(2)]
-        h_norm = [torch.zeros(8, dtype=torch.float64, pin_memory=True) for _ in range(2)]
-        solvers = [(J, coord, stream), (J2, coord2, stream2)]
+        h_out = [torch.empty(slab_elems, dtype=torch.float32, pin_memory=True) for _ in range(S)]
+        h_norm = [torch.zeros(8, dtype=torch.float64, pin_memory=True) for _ in range(S)]
 
         def e2e_step(i, pipelined):
-            Jx, cx, _ = solvers[i % 2] if pipelined else solvers[0]
-            b = i % 2 if pipelined else 0
+            b = i % S if pipelined else 0
+            Jx, cx, _ = solvers[b]
             Jx.copy_in_async(cx, h_in.data_ptr())
             Jx.run(cx, ips, a.norm_every, use_graph, norms_out=h_norm[b].numpy())
             Jx.copy_out_async(cx, h_out[b].data_ptr())
 
         for pipelined in (False, True):  # warm-up (graph builds are collective and synchronous)
-            for i in range(2):
+            for i in range(S):
                 e2e_step(i, pipelined)
-        coord.sync()
-        coord2.sync()
+        for _, cx, _ in solvers:
+            cx.sync()
         times = {}
         for pipelined in (False, True):
             barrier(dist)
             torch.cuda.synchronize()
             f0 = torch.cuda.Event(enable_timing=True)
             f0.record(stream)
-            stream2.wait_event(f0)
+            for _, _, sx in solvers[1:]:
+                sx.wait_event(f0)
             for i in range(ke):
                 e2e_step(i, pipelined)
-            f1, f2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            f1.record(stream)
-            f2.record(stream2)
-            coord.sync()
-            coord2.sync()
+            ends = []
+            for _, _, sx in solvers:
+                f = torch.cuda.Event(enable_timing=True)
+                f.record(sx)
+                ends.append(f)
+            for _, cx, _ in solvers:
+                cx.sync()
             barrier(dist)
-            times[pipelined] = allreduce_max(dist, max(f0.elapsed_time(f1), f0.elapsed_time(f2)))
+            times[pipelined] = allreduce_max(dist, max(f0.elapsed_time(f) for f in ends))
         te, ts = times[True], times[False]
         e2e = {"value": round(pts_rank * world * ips * ke / (te / 1e3) / 1e9, 3), "unit": UNIT,
                "h2d_bytes_per_step": slab_elems * 4, "d2h_bytes_per_step": slab_elems * 4 + 8 * (len(range(0, ips, a.norm_every)) if a.norm_every > 0 else 0),
                "steps": ke, "ms_per_step": round(te / ke, 3),
-               "pipeline": "2 solvers on 2 streams alternate steps (H2D of step i+1 overlaps compute + D2H of step i)",
+               "pipeline": f"{S} solvers on {S} streams take turns (step i+1's H2D overlaps step i's compute and D2H)",
                "serial_value": round(pts_rank * world * ips * ke / (ts / 1e3) / 1e9, 3),
                "serial_ms_per_step": round(ts / ke, 3)}
         comm.barrier()
-        J2.destroy()
-        coord2.destroy()
+        for Jx, cx, _ in solvers[1:]:
+            Jx.destroy()
+            cx.destroy()
 
     comm.barrier()
     J.destroy()
