@@ -24,6 +24,28 @@ static __device__ unsigned long long* uc_trace_ptr;
   } while (0)
 #endif
 
+// Bounds checks of the T-level kernel's geometry (build.py --define UC_DEBUG_CHECKS=1 --out ...):
+// compute-sanitizer is not available on the GPU pool, so a debug build asserts what the
+// kernel's memory safety rests on (rows read and written, ring offsets, balanced tables) and
+// traps on the first violation.  Off in the product.
+#ifndef UC_DEBUG_CHECKS
+#define UC_DEBUG_CHECKS 0
+#endif
+#if UC_DEBUG_CHECKS
+#define UC_CHECK(cond)                                                                          \
+  do {                                                                                         \
+    if (!(cond)) {                                                                             \
+      printf("UC_CHECK failed: %s (block %d thread %d, %s:%d)\n", #cond, blockIdx.x, threadIdx.x, \
+             __FILE__, __LINE__);                                                              \
+      __trap();                                                                                \
+    }                                                                                          \
+  } while (0)
+#else
+#define UC_CHECK(cond) \
+  do {                 \
+  } while (0)
+#endif
+
 // System-scope fence before the release-store of a round's flag to a neighbour on another GPU
 // (A/B: 0 relies on st.release.sys cumulativity after the block barrier alone)
 #ifndef UC_ROUND_SYS_FENCE
@@ -571,6 +593,7 @@ __device__ __forceinline__ bool march_t(const JacobiParams& p, const float* src,
       const int right = min(xe + PAD, p.nx);
       const unsigned bytes = (unsigned)(right - left) * 4u;
       const int off = left - (xs - PAD);
+      UC_CHECK(off >= 0 && off + (int)(bytes / 4) <= ST && (bytes & 15u) == 0u && NS * ST * 4 + 128 <= 200 * 1024);
 #if UC_L2_EVICT_FIRST
       const uint64_t pol = policy_evict_first();
 #else
@@ -698,6 +721,12 @@ __device__ __forceinline__ double t_body(const JacobiParams& p, uint64_t k, int 
   UC_TRACE_AT(1);
   const int a = deep_top ? lo : max(lo, PT + 1);
   const int b = deep_bot ? hi : min(hi, p.n - PT);
+  UC_CHECK(s >= 0 && s < p.strips && q >= 0 && q < p.chunks && lo >= 1 && hi <= p.n);
+  // the march streams A_k rows a-T .. b+T: only a first/last chunk (which waited for the halo
+  // flags in round 1, or holds a deep halo) may reach row 0 / n+1 and beyond
+  UC_CHECK(a > b || a - T >= (deep_top ? 1 - T : top_blk ? 0 : 1));
+  UC_CHECK(a > b || b + T <= (deep_bot ? p.n + T : bot_blk ? p.n + 1 : p.n));
+  UC_CHECK((int)threadIdx.x >= p.consumers || !g.in_grid || g.ring_off + 4 <= kStageFloats<G>);  // consumers
   if (a <= b) {
     // fixed columns (0, NX-1) among the block's lanes, ghosts included: keep them fixed
     const int xs4 = s * p.strip4;
@@ -812,6 +841,8 @@ static __device__ __noinline__ void bal_resize(const JacobiParams& p, unsigned c
       const long long B = q == Q - 1 ? E : (long long)floor(cum + 1e-6);
       const int lo = 1 + (int)max(0LL, min(prev - p.chunk_shrink, (long long)p.n));
       const int hi = (int)max(0LL, min(B - p.chunk_shrink, (long long)p.n));
+      UC_CHECK(B >= prev && lo <= hi + 1 && (q == 0 ? lo == 1 : true) && (q == Q - 1 ? hi == p.n : true));
+      UC_CHECK(q == 0 || q == Q - 1 || hi - lo + 1 >= p.bal_levels);
       p.bal_tab[p.bal_inv[s * Q + q]] = make_int4(s, q, lo, hi);
       prev = B;
     }
