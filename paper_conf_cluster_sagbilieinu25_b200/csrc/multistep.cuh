@@ -244,6 +244,52 @@ __device__ __forceinline__ float4 row2_update_natural(const Row2& up, const Row2
   return o;
 }
 
+// Level 1 from natural-order rows (UC_LEVEL1_NATURAL, T >= 2): the A_k rows stay in the pairs
+// the ring load lands them in, (x0, x1) | (x2, x3), and level 1 forms its sums with scalar adds
+// written straight into the frame's pairs -- 8 FADD + 2 FADD2 instead of four permuting adds
+// per row plus 8 packed FP32 instructions (the same IEEE operations on the same operands).
+#ifndef UC_LEVEL1_NATURAL
+#define UC_LEVEL1_NATURAL 1
+#endif
+__device__ __forceinline__ Row2 nat_row2(float4 n) { return Row2{pk2(n.x, n.y), pk2(n.z, n.w)}; }
+__device__ __forceinline__ float4 nat_float4(const Row2& r) {
+  float4 n;
+  upk2(r.p, n.x, n.y);
+  upk2(r.q, n.z, n.w);
+  return n;
+}
+__device__ __forceinline__ pair_t nat_lr(const Row2& c) {
+  float x0, x1, x2, x3;
+  upk2(c.p, x0, x1);
+  upk2(c.q, x2, x3);
+  (void)x1;
+  (void)x2;
+  return pk2(__shfl_up_sync(kFull, x3, 1), __shfl_down_sync(kFull, x0, 1));
+}
+template <bool DIRI, bool SC>
+__device__ __forceinline__ Row2 row2_update_nat_in(const Row2& up, const Row2& c, const Row2& dn, pair_t lr, int x4,
+                                                   int nx4) {
+  float u0, u1, u2, u3, c0, c1, c2, c3, d0, d1, d2, d3, L, R;
+  upk2(up.p, u0, u1);
+  upk2(up.q, u2, u3);
+  upk2(c.p, c0, c1);
+  upk2(c.q, c2, c3);
+  upk2(dn.p, d0, d1);
+  upk2(dn.q, d2, d3);
+  upk2(lr, L, R);
+  const pair_t hp = pk2(__fadd_rn(L, c1), __fadd_rn(c2, R));   // (h0, h3)
+  const pair_t hq = pk2(__fadd_rn(c0, c2), __fadd_rn(c1, c3));  // (h1, h2)
+  const pair_t vp = pk2(__fadd_rn(u0, d0), __fadd_rn(u3, d3));
+  const pair_t vq = pk2(__fadd_rn(u1, d1), __fadd_rn(u2, d2));
+  Row2 o{SC ? f2add(hp, vp) : f2quarter(f2add(hp, vp)), SC ? f2add(hq, vq) : f2quarter(f2add(hq, vq))};
+  if (DIRI) {
+    float a0, a3;
+    upk2(o.p, a0, a3);
+    o.p = pk2(x4 == 0 ? c0 : a0, x4 == nx4 - 1 ? c3 : a3);
+  }
+  return o;
+}
+
 struct GhostLayout {
   int x4;        // float4 column of this thread (ghost lanes: the neighbour's edge column)
   bool in_grid;  // 0 <= x4 < nx4 (may be loaded)
@@ -484,10 +530,12 @@ __device__ __forceinline__ bool range_ok(const RowRange& r) {
 // row (STORE: from the 2T-th row on).  The horizontal neighbours of every level's middle row
 // (w1[j], known before the step's new row arrives) are shuffled up front, off the level chain
 // (new row -> level 1 -> ... -> level T); the first HOIST levels' before the ring wait.
+template <int T>
+constexpr bool kNat0 = UC_LEVEL1_NATURAL && T >= 2;  // level-0 rows in natural pairs
 template <int T, int J0, int J1>
 __device__ __forceinline__ void t_neighbours2(const Row2 (&w1)[T], pair_t (&lr)[T]) {
 #pragma unroll
-  for (int j = J0; j < J1; ++j) lr[j] = row2_lr(w1[j]);
+  for (int j = J0; j < J1; ++j) lr[j] = (kNat0<T> && j == 0) ? nat_lr(w1[j]) : row2_lr(w1[j]);
 }
 template <int T, int NL, bool DIRI, bool STORE, bool SC>
 __device__ __forceinline__ void t_levels2(const Row2& n0, const GhostLayout& g, int nx4, int a, int b, int i,
@@ -497,10 +545,12 @@ __device__ __forceinline__ void t_levels2(const Row2& n0, const GhostLayout& g, 
   Row2 nv = n0;
 #pragma unroll
   for (int j = 0; j < T - 1; ++j) {
-    const Row2 o = row2_update<DIRI, SC>(w0[j], w1[j], nv, lr[j], g.x4, nx4);  // level j+1, row r-j-1
+    const bool nat = kNat0<T> && j == 0;  // level 1 from natural-order A_k rows
+    const Row2 o = nat ? row2_update_nat_in<DIRI, SC>(w0[j], w1[j], nv, lr[j], g.x4, nx4)
+                       : row2_update<DIRI, SC>(w0[j], w1[j], nv, lr[j], g.x4, nx4);  // level j+1, row r-j-1
     if (NL == j + 1 && g.own) {
       const int y = a - T + i - j - 1;
-      if (y >= a && y <= b) acc_sq(acc, from_row2(o), from_row2(w1[j]));
+      if (y >= a && y <= b) acc_sq(acc, from_row2(o), nat ? nat_float4(w1[j]) : from_row2(w1[j]));
     }
     w0[j] = w1[j];
     w1[j] = nv;
@@ -528,7 +578,7 @@ __device__ __forceinline__ void t_step2(const float* ring, uint64_t* full, uint6
   t_neighbours2<T, 0, HOIST>(w1, lr);
   const float4 n = t_fetch(ring, full, empty, ST, NS, g, cur);
   if (SC) range_add(rng, n);
-  const Row2 nv = ring_row2<DIRI>(n);
+  const Row2 nv = kNat0<T> ? nat_row2(n) : ring_row2<DIRI>(n);
   t_neighbours2<T, HOIST, T>(w1, lr);
   t_levels2<T, NL, DIRI, STORE, SC>(nv, g, nx4, a, b, i, w0, w1, lr, out, pitch, acc);
 }
@@ -553,7 +603,7 @@ __device__ __forceinline__ void t_group2(const float* ringp, uint64_t* full, uin
 #endif
     const float4 n = *reinterpret_cast<const float4*>(ringp + u * ST);
     if (SC) range_add(rng, n);
-    const Row2 nv = ring_row2<DIRI>(n);
+    const Row2 nv = kNat0<T> ? nat_row2(n) : ring_row2<DIRI>(n);
     __syncwarp();
     mbar_arrive_if(empty + u, lane0);
 #if UC_RING_TEST_AHEAD
